@@ -1,0 +1,323 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 corner-force path (BASELINE.json metric: corner-force zones/s and FP64 GFLOP/s,
+3D Sedov Q4-Q3 32^3 = config C4, at 1/2/4/8 B200).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config C4]
+
+A step = one full corner-force evaluation (all §8(a) rows: gather, geometry, viscosity, EOS/stress,
+back contractions, deterministic F.1 gather, F^T v, min dt [+ the NCCL shared-DOF exchange for N>1])
+over the whole mesh.  N>1 (torchrun): the fixed C4 mesh is block-partitioned over the ranks (strong
+scaling), each rank times its own evals on its stream, the max over ranks is reported.
+
+--impl reference times the CPU oracle (the paper has no runnable code) on a bounded
+sample of the same workload on this host's cores.
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "corner-force zones/s & FP64 GFLOP/s (Q4-Q3 3D Sedov) at 1/2/4/8 B200"
+# FP64 ALU roofline: 148 SMs x 64 FP64 FMA/clk x 2 flop x 1.965 GHz (B200_PROFILING.md SM count and
+# max clock; 64 FP64 FMA/clk/SM from the measured P0 microbenchmark, profiles/r01_p0_fp64_peaks.json:
+# DFMA 34.2 TF, DMMA 37.1 TF at 1965 MHz).  DESIGN.md §5.
+FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12
+
+
+def env_rank():
+    return int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("LOCAL_RANK", "0"))
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled DURING the timed region (B200_PROFILING.md)."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.gpu = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, smax, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            p = [x.strip() for x in ln.split(",")]
+            if len(p) < 8:
+                continue
+            try:
+                sm.append(float(p[1]))
+                smax = max(smax, float(p[2]))
+            except ValueError:
+                continue
+            for nm, val in zip(names, p[4:8]):
+                if val.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": smax, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def workload_desc(name):
+    import synth
+    c = synth.CONFIGS[name]
+    return c["desc"]
+
+
+def load_traffic():
+    """dram bytes per KB1 launch from the committed ncu --set full summary (or None)."""
+    p = os.path.join(ROOT, "profiles", "kb1_ncu_summary.json")
+    try:
+        d = json.load(open(p))
+        return d.get("dram_bytes_per_launch"), d.get("source")
+    except Exception:
+        return None, None
+
+
+def oracle_sample(mesh, st, seconds=15.0, max_zones=None):
+    """Time the oracle (as it stands) on a bounded, contiguous sample of the workload's zones."""
+    import oracle
+    h0 = (float(np.prod(mesh.L)) / mesh.num_zones) ** (1.0 / mesh.dim) / mesh.order
+    par = oracle.Params(h0=h0)
+    nthr = oracle.max_threads()
+    # calibrate on a small sample, then size the sample for ~`seconds`
+    nz = max(nthr, 16)
+    t0 = time.perf_counter()
+    oracle.evaluate(mesh, st, params=par, zones=np.arange(nz), assemble=False)
+    t1 = time.perf_counter() - t0
+    nz2 = int(min(mesh.num_zones, max(nz, seconds / max(t1, 1e-6) * nz)))
+    if max_zones:
+        nz2 = min(nz2, max_zones)
+    t0 = time.perf_counter()
+    oracle.evaluate(mesh, st, params=par, zones=np.arange(nz2), assemble=True)
+    t = time.perf_counter() - t0
+    return nz2, t, nthr
+
+
+def run_reference(args):
+    rank, world, _ = env_rank()
+    if rank != 0:
+        return 0
+    import synth
+    mesh, st = synth.config(args.config, args.state)
+    times = []
+    nz = None
+    for i in range(args.warmup + args.steps):
+        n, t, nthr = oracle_sample(mesh, st, seconds=args.cpu_seconds / max(args.steps, 1), max_zones=nz)
+        nz = n
+        if i >= args.warmup:
+            times.append(t)
+    tot = sum(times)
+    value = nz * len(times) / tot
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "zones/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / len(times), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{args.config}: {workload_desc(args.config)}", "state": args.state,
+                   "zones": mesh.num_zones},
+        "cpu_baseline": {"value": value, "unit": "zones/s", "cores": nthr, "kind": "oracle",
+                         "sample": f"first {nz} of {mesh.num_zones} zones per step (plain C oracle, OpenMP over zones)"},
+        "e2e": {"value": value, "unit": "zones/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line))
+    return 0
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    import synth
+
+    rank, world, local = env_rank()
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    mesh, st = synth.config(args.config, args.state)
+    Zg = mesh.num_zones
+    part = None
+    uid = None
+    if world > 1:
+        parts = synth.partition(mesh, world)
+        part = parts[rank]
+        obj = [cf.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+        lmesh, lst = part.local_mesh(mesh), part.local_state(st)
+    else:
+        lmesh, lst = mesh, st
+    stream = torch.cuda.Stream(device=dev)
+    with torch.cuda.stream(stream):
+        h = cf.from_synth(mesh, part=part, nccl_uid=uid, stream=stream) if world > 1 else cf.from_synth(lmesh, stream=stream)
+    info = h.info
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(dev)
+    x, v, e, r = t(lst.x), t(lst.v), t(lst.e), t(lst.rho0detJ0)
+    out = h.alloc_outputs()
+    in_bytes = sum(a.numel() * 8 for a in (x, v, e, r))
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    # warm-up
+    for _ in range(args.warmup):
+        h.eval(x, v, e, r, out=out)
+    barrier()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local if world > 1 else 0) as clk:
+        ev0.record(stream)
+        for _ in range(args.steps):
+            h.eval(x, v, e, r, out=out)
+        ev1.record(stream)
+        barrier()
+    ms = ev0.elapsed_time(ev1)
+    if world > 1:
+        tt = torch.tensor([ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms = float(tt.item())
+    ms_step = ms / args.steps
+    value = Zg * args.steps / (ms / 1e3)
+
+    # per-kernel breakdown (separate pass, events on the library's stream)
+    h.set_timing(True)
+    kb = np.zeros(3)
+    nkt = max(args.steps, 5)
+    for _ in range(nkt):
+        h.eval(x, v, e, r, out=out)
+        kb += np.array(h.kernel_times())
+    h.set_timing(False)
+    kb /= nkt
+    kb1_ms = float(kb[0])
+    Zl = lmesh.num_zones
+    flops_eval_local = info["flops_per_zone"] * Zl
+    achieved_tf = flops_eval_local / (kb1_ms / 1e3) / 1e12
+    gflops_total = info["flops_per_zone"] * Zg / (ms_step / 1e3) / 1e9
+    traffic, tsrc = load_traffic()
+
+    # e2e through the public API with host buffers (pinned), H2D + eval + D2H inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        hx = [torch.from_numpy(np.ascontiguousarray(a)).pin_memory() for a in (lst.x, lst.v, lst.e, lst.rho0detJ0)]
+        ho = (torch.empty(tuple(out[0].shape), dtype=torch.float64).pin_memory(),
+              torch.empty(tuple(out[1].shape), dtype=torch.float64).pin_memory(),
+              torch.empty(1, dtype=torch.float64).pin_memory())
+        h.eval_host(*hx, out=ho)
+        barrier()
+        k2 = max(3, min(args.steps, 10))
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a0.record(stream)
+        for _ in range(k2):
+            h.eval_host(*hx, out=ho)
+        a1.record(stream)
+        barrier()
+        ems = a0.elapsed_time(a1)
+        if world > 1:
+            tt = torch.tensor([ems], device=dev, dtype=torch.float64)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            ems = float(tt.item())
+        out_bytes = sum(o.numel() * 8 for o in ho)
+        e2e = {"value": Zg * k2 / (ems / 1e3), "unit": "zones/s", "h2d_bytes_per_step": int(in_bytes),
+               "d2h_bytes_per_step": int(out_bytes), "ms_per_step": ems / k2}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        nz, tc, nthr = oracle_sample(mesh, st, seconds=args.cpu_seconds)
+        cpu = {"value": nz / tc, "unit": "zones/s", "cores": nthr, "kind": "oracle",
+               "sample": f"first {nz} of {Zg} zones of the same C4 S1 state, one evaluation (plain C oracle, "
+                         f"OpenMP over zones, serial assembly), {tc:.1f} s"}
+
+    if rank == 0:
+        clocks = clk.summary()
+        line = {
+            "metric": METRIC, "value": value, "unit": "zones/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"{args.config}: {workload_desc(args.config)}", "state": args.state,
+                       "zones": Zg, "order": mesh.order, "dim": mesh.dim,
+                       "parallelism": f"domain decomposition {synth.block_dims(mesh.dim, world)}" if world > 1 else "single GPU",
+                       "l2": f"inputs larger than L2 ({in_bytes / 1e6:.0f} MB of inputs per rank + "
+                             f"{Zl * info['nk'] * mesh.dim * 8 / 1e6:.0f} MB zone-local buffer vs 126 MB L2); no flush"},
+            "gflops": gflops_total,
+            "roofline": {"bound": "alu", "achieved": achieved_tf, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
+                         "frac": achieved_tf / FP64_PEAK_TFLOPS, "traffic": traffic,
+                         "kernel": "kb1_corner_force_3d" if mesh.dim == 3 else "kb1_corner_force_2d",
+                         "kernel_ms": kb1_ms, "kb2_ms": float(kb[1]), "exchange_ms": float(kb[2]),
+                         "flops_per_zone": info["flops_per_zone"],
+                         "peak_note": "FP64 ALU: 148 SM x 64 FMA/clk x 2 x 1.965 GHz (measured DFMA 34.2 / DMMA 37.1 TF)",
+                         "traffic_source": tsrc},
+            "e2e": e2e,
+            "gpu_launches": int(info["kernels_per_eval"] * args.steps),
+            "clocks": clocks,
+            "cpu_baseline": cpu,
+            "launch": {k: info[k] for k in ("zones_per_cta", "threads_per_cta", "num_ctas", "smem_bytes",
+                                            "regs_per_thread", "local_bytes")},
+        }
+        print(json.dumps(line))
+    h.close()
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C4")
+    ap.add_argument("--state", default="S1")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

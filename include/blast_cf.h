@@ -1,0 +1,159 @@
+/*
+ * blast_cf.h — C ABI of the B200-native BLAST corner-force library (libblastcf.so).
+ *
+ * The library evaluates, for Q_k-Q_{k-1} finite elements in 2D and 3D and in FP64, the generalized
+ * corner force of BLAST's semi-discrete Lagrangian hydrodynamics (§2, eqs (1)-(6))
+ * and returns only the right-hand sides the time integrator needs (§3.1.2: "we avoid
+ * transferring the full matrix F"):
+ *
+ *   out_Fdot1   = F . 1           assembled into global kinematic DOFs   (momentum RHS is -F.1, eq (1);
+ *                                                                         kernel 8)
+ *   out_FTv     = F_z^T . v_z     per zone                               (energy RHS before M_E^{-1}, eq (2);
+ *                                                                         kernel 10)
+ *   out_dt_min  = min over zones and quadrature points of the time-step estimate
+ *                                                     (steps 4.2 and 5; MPI min 797-798)
+ *
+ * with (F_z)_{ij} = sum_k alpha_k sigma(q_k) : J_z^{-1}(q_k) grad W_i(q_k) phi_j(q_k) |J_z(q_k)|  (eq (4)),
+ * factored F_z = A_z B^T (eqs (5)-(6)).  The stress sigma (EOS + artificial viscosity, "see [1]",
+ * PAPER.md:276-280) and the time-step formula follow the readings in DESIGN.md §3.
+ *
+ * Conventions (all arrays FP64 unless noted; "x fastest" lexicographic orderings):
+ *   reference element [0,1]^dim; kinematic basis: tensor Lagrange on the k+1 Gauss-Lobatto-Legendre
+ *   points; thermodynamic basis: tensor Bernstein of degree k-1; quadrature: tensor Gauss-Legendre with
+ *   2k points per direction.  Nk = (k+1)^dim, Nt = k^dim, Nq = (2k)^dim.
+ *
+ * Errors: every function returns BLAST_CF_OK (0) or a positive code; blast_cf_error_string() names it
+ * and blast_cf_last_error() gives a message for the most recent failure on the calling thread.
+ * Asynchronous CUDA faults in an eval surface as BLAST_CF_ECUDA at the next call on the handle.
+ */
+#ifndef BLAST_CF_H
+#define BLAST_CF_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+  BLAST_CF_OK = 0,
+  BLAST_CF_EINVAL = 1,       /* null / inconsistent argument */
+  BLAST_CF_EUNSUPPORTED = 2, /* dim/order outside {2,3} x [1,8], or non-affine initial zones with viscosity on */
+  BLAST_CF_ENOMEM = 3,       /* device or host allocation failed */
+  BLAST_CF_ECUDA = 4,        /* CUDA runtime error (launch or asynchronous fault) */
+  BLAST_CF_ENCCL = 5         /* NCCL error in the multi-GPU shared-DOF exchange */
+};
+
+typedef struct blast_cf blast_cf; /* opaque; owns tables, maps, workspace and (nranks > 1) the NCCL comm */
+
+/* The mesh as seen by ONE rank (§3.4: each MPI task owns a sub-domain).
+ * All pointers are HOST pointers; the library copies what it needs at create and keeps no reference. */
+typedef struct {
+  int32_t dim;               /* 2 or 3 */
+  int32_t order;             /* k in [1, 8]: Q_k kinematic, Q_{k-1} thermodynamic */
+  int64_t num_zones;         /* zones on this rank */
+  int64_t num_nodes;         /* kinematic nodes touched by this rank's zones */
+  const int32_t *zone_nodes; /* [num_zones][Nk] local node ids, local node a = l0 + (k+1)(l1 + (k+1) l2) */
+  const double *x0;          /* [dim][num_nodes] initial node positions (J0, h0 of the viscosity) */
+  const int32_t *zone_mat;   /* [num_zones] material id, or NULL (all material 0) */
+  const double *mat_gamma;   /* [num_mats] ideal-gas gamma per material */
+  int32_t num_mats;
+  /* domain decomposition (nranks == 1: single GPU, the fields below are ignored) */
+  int32_t rank, nranks;
+  int32_t num_neighbors;     /* ranks sharing at least one node with this rank */
+  const int32_t *nbr_rank;   /* [num_neighbors] ascending */
+  const int64_t *nbr_offset; /* [num_neighbors + 1] */
+  const int32_t *nbr_nodes;  /* [nbr_offset[num_neighbors]] local node ids shared with nbr_rank[i],
+                                ordered by global node id (identical order on both sides) */
+} blast_cf_mesh;
+
+/* Method constants (DESIGN.md §3 readings R8, R10, R11). */
+typedef struct {
+  double cfl;            /* 0.5 */
+  double q_quad;         /* 2.0  quadratic viscosity coefficient */
+  double q_lin;          /* 0.5  linear viscosity coefficient */
+  double eps_switch;     /* 1e-12 compression-switch width */
+  double h0;             /* <= 0: computed at create as (V_global / Z_global)^(1/dim) / k */
+  int32_t use_viscosity; /* 1 */
+  int32_t use_vorticity; /* 1: psi0 = |div v| / |grad v|_F, else 1 */
+} blast_cf_params;
+
+void blast_cf_default_params(blast_cf_params *p);
+
+/* Create a handle.  `order` and `dim` must equal mesh->order / mesh->dim (the north-star call shape
+ * blast_cf_create(mesh, order, dim)).  params NULL = defaults.  cuda_stream: a cudaStream_t (NULL =
+ * the legacy default stream) on which every eval is enqueued.  nccl_unique_id: pointer to an
+ * ncclUniqueId (128 bytes) shared by all ranks when mesh->nranks > 1, else NULL; the caller must have
+ * selected this rank's CUDA device.  All device memory is allocated here; eval never allocates. */
+int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_cf_params *params,
+                    void *cuda_stream, const void *nccl_unique_id, blast_cf **out);
+
+/* One corner-force evaluation.  All seven arrays are DEVICE pointers owned by the caller:
+ *   x, v        [dim][num_nodes]  current positions and velocities (SoA)
+ *   e           [num_zones][Nt]   specific internal energy, Bernstein coefficients
+ *   rho0detJ0   [num_zones][Nq]   rho0(q) * det J0(q) at the quadrature points (no quadrature weight)
+ *   out_Fdot1   [dim][num_nodes]  +F.1 (the momentum RHS is -F.1); on shared nodes every sharing rank
+ *                                 holds the fully summed value (summed in ascending rank order)
+ *   out_FTv     [num_zones][Nt]   F_z^T v_z
+ *   out_dt_min  [1]               global min dt; +inf if no point has a positive inverse dt; 0 if any
+ *                                 det J <= 0 (inverted zone)
+ * Inputs are read-only, outputs are overwritten.  Enqueues on the handle's stream and returns without
+ * synchronizing (CUDA-graph capturable for nranks == 1).  Not thread-safe per handle. */
+int blast_cf_eval(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                  double *out_Fdot1, double *out_FTv, double *out_dt_min);
+
+/* Same evaluation with HOST buffers (pinned memory recommended): copies the inputs host->device,
+ * evaluates, copies the three outputs back and synchronizes the stream before returning.  Device
+ * staging buffers are allocated by the first call and reused. */
+int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                       double *out_Fdot1, double *out_FTv, double *out_dt_min);
+
+/* Tests only: the zone-local corner force matrices F_z = A_z B^T ([num_zones][dim*Nk][Nt], device), as
+ * formed by kernel 7 of the paper.  Production eval never forms them. */
+int blast_cf_eval_debug_Fz(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                           double *out_Fz);
+
+typedef struct {
+  int32_t dim, order, nq, nk, nt;
+  int64_t num_zones, num_nodes;
+  double h0;                  /* the length scale in use */
+  int32_t zones_per_cta, threads_per_cta, num_ctas, smem_bytes, regs_per_thread, local_bytes;
+  double flops_per_zone;      /* algorithmic FP64 flops per zone (DESIGN.md §5 model) */
+  double alg_bytes;           /* algorithmic HBM bytes per eval */
+  int32_t kernels_per_eval;   /* CUDA kernels launched by one eval */
+} blast_cf_info;
+
+int blast_cf_get_info(const blast_cf *h, blast_cf_info *info);
+
+/* Per-kernel timing for the roofline report: when enabled, each eval records CUDA events around its
+ * kernels on the handle's stream.  blast_cf_kernel_times() synchronizes on the last eval and returns the
+ * milliseconds of [0] the corner-force kernel (KB1), [1] the node gather + dt (KB2), [2] the exchange
+ * (nranks > 1, else 0) of that eval. */
+int blast_cf_set_timing(blast_cf *h, int enable);
+int blast_cf_kernel_times(blast_cf *h, float *ms3);
+
+/* Tests only: the per-CTA minimum dt of the last eval (CTA c covers zones [c*zpc, (c+1)*zpc)), copied
+ * to host_out[capacity] after synchronizing the stream.  host_out NULL: only report the sizes. */
+int blast_cf_debug_cta_dt(blast_cf *h, double *host_out, int64_t capacity, int32_t *num_ctas, int32_t *zones_per_cta);
+
+int blast_cf_destroy(blast_cf *h);
+const char *blast_cf_error_string(int code);
+const char *blast_cf_last_error(void);
+
+/* Host-only (no GPU needed), for the multi-rank tests: the exchange plan the library builds from a
+ * rank's neighbour lists.  Row r of the pack buffers is the partial F.1 of nbr_nodes[r].  For every
+ * shared node unique_nodes[u] (ascending local id) the partials are summed in the order
+ * src[src_ptr[u] .. src_ptr[u+1]) — ascending rank — where src >= 0 is this rank's own partial (send
+ * row src) and src < 0 a neighbour's (recv row -src-1).  capacity bounds unique_nodes/src_ptr/src. */
+int blast_cf_exchange_plan(int32_t rank, int32_t num_neighbors, const int32_t *nbr_rank, const int64_t *nbr_offset,
+                           const int32_t *nbr_nodes, int64_t capacity, int64_t *num_unique, int32_t *unique_nodes,
+                           int64_t *src_ptr, int64_t *src);
+
+/* Size of ncclUniqueId (bytes) and a helper so Python can create it without linking NCCL itself. */
+int blast_cf_nccl_unique_id_size(void);
+int blast_cf_nccl_get_unique_id(void *out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BLAST_CF_H */

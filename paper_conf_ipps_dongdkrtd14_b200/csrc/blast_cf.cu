@@ -1,0 +1,637 @@
+// libblastcf.so — host library and C ABI (include/blast_cf.h) of the B200 corner-force path.
+//
+// create(): validates the mesh, builds the 1-D tables (tables.h), the per-zone J0^{-1} of the affine
+// initial zones and h0, the inverse node -> (zone, local) CSR in ascending zone id, uploads everything
+// and sizes the launch.  eval(): KB1 (kb1_corner_force.cuh) then KB2 (kb2_gather.cuh) on the handle's
+// stream, plus the shared-DOF exchange when nranks > 1 (exchange.cuh).  No allocation in eval.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/blast_cf.h"
+#include "kb1_corner_force.cuh"
+#include "kb2_gather.cuh"
+#include "tables.h"
+#include "exchange.cuh"
+
+namespace {
+
+thread_local std::string g_last_error;
+
+int fail(int code, const char *fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_last_error = buf;
+  return code;
+}
+
+#define CUDA_TRY(expr)                                                                       \
+  do {                                                                                       \
+    cudaError_t e_ = (expr);                                                                 \
+    if (e_ != cudaSuccess)                                                                   \
+      return fail(e_ == cudaErrorMemoryAllocation ? BLAST_CF_ENOMEM : BLAST_CF_ECUDA,        \
+                  "%s: %s (%s:%d)", #expr, cudaGetErrorString(e_), __FILE__, __LINE__);      \
+  } while (0)
+
+template <typename T>
+int upload(T **dst, const T *src, size_t count) {
+  CUDA_TRY(cudaMalloc((void **)dst, std::max<size_t>(count, 1) * sizeof(T)));
+  if (count) CUDA_TRY(cudaMemcpy(*dst, src, count * sizeof(T), cudaMemcpyHostToDevice));
+  return BLAST_CF_OK;
+}
+
+// ------------------------------------------------------------------------------------------------
+// kernel instantiation table: (dim, k) -> zones per CTA, threads, shared memory, launcher
+// ------------------------------------------------------------------------------------------------
+typedef void (*kb1_launch_fn)(const KB1Args &, int grid, cudaStream_t);
+
+struct KB1Variant {
+  int zpc, nth, smem;
+  kb1_launch_fn launch;
+  const void *func;
+};
+
+template <int K, int ZPC, int MINB>
+void launch3(const KB1Args &a, int grid, cudaStream_t s) {
+  using C = KB1Cfg3<K, ZPC>;
+  kb1_corner_force_3d<K, ZPC, MINB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+}
+template <int K, int ZPC, int MINB>
+void launch2(const KB1Args &a, int grid, cudaStream_t s) {
+  using C = KB1Cfg2<K, ZPC>;
+  kb1_corner_force_2d<K, ZPC, MINB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+}
+template <int K, int ZPC, int MINB>
+KB1Variant variant3() {
+  using C = KB1Cfg3<K, ZPC>;
+  return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3<K, ZPC, MINB>,
+                    (const void *)&kb1_corner_force_3d<K, ZPC, MINB>};
+}
+template <int K, int ZPC, int MINB>
+KB1Variant variant2() {
+  using C = KB1Cfg2<K, ZPC>;
+  return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch2<K, ZPC, MINB>,
+                    (const void *)&kb1_corner_force_2d<K, ZPC, MINB>};
+}
+
+KB1Variant select_variant(int dim, int k) {
+  if (dim == 3) {
+    switch (k) {
+      case 1: return variant3<1, 32, 2>();
+      case 2: return variant3<2, 16, 2>();
+      case 3: return variant3<3, 8, 2>();
+      case 4: return variant3<4, 4, 2>();
+      case 5: return variant3<5, 2, 2>();
+      case 6: return variant3<6, 2, 1>();
+      case 7: return variant3<7, 1, 2>();
+      case 8: return variant3<8, 1, 1>();
+    }
+  } else {
+    switch (k) {
+      case 1: return variant2<1, 64, 2>();
+      case 2: return variant2<2, 16, 2>();
+      case 3: return variant2<3, 8, 2>();
+      case 4: return variant2<4, 4, 2>();
+      case 5: return variant2<5, 2, 2>();
+      case 6: return variant2<6, 2, 2>();
+      case 7: return variant2<7, 1, 2>();
+      case 8: return variant2<8, 1, 2>();
+    }
+  }
+  return KB1Variant{0, 0, 0, nullptr, nullptr};
+}
+
+// Debug: F_z = A_z B^T from S(q) (kernel 7 of the paper); one CTA per zone.
+template <int D>
+__global__ void kbd_form_Fz(const double *Sq, const double *tab, int k, int64_t Z, double *Fz) {
+  const int n = 2 * k, p = k + 1, t = k;
+  const int nk = D == 3 ? p * p * p : p * p, nt = D == 3 ? t * t * t : t * t, nq = D == 3 ? n * n * n : n * n;
+  const double *B = tab, *G = tab + n * p, *Phi = tab + 2 * n * p;
+  const int64_t z = blockIdx.x;
+  if (z >= Z) return;
+  for (int i = threadIdx.x; i < D * nk * nt; i += blockDim.x) {
+    const int row = i / nt, j = i - row * nt;
+    const int c = row / nk, a = row - c * nk;
+    int ai[3] = {a % p, (a / p) % p, a / (p * p)};
+    int ji[3] = {j % t, (j / t) % t, j / (t * t)};
+    double s = 0.0;
+    for (int q = 0; q < nq; ++q) {
+      int qi[3] = {q % n, (q / n) % n, q / (n * n)};
+      double phi = 1.0;
+      for (int d = 0; d < D; ++d) phi *= Phi[qi[d] * t + ji[d]];
+      double acc = 0.0;
+      for (int d = 0; d < D; ++d) {
+        double dw = 1.0;
+        for (int e = 0; e < D; ++e) dw *= (e == d ? G : B)[qi[e] * p + ai[e]];
+        acc += Sq[(z * nq + q) * D * D + c * D + d] * dw;
+      }
+      s += acc * phi;
+    }
+    Fz[(z * D * nk + row) * nt + j] = s;
+  }
+}
+
+}  // namespace
+
+
+// ------------------------------------------------------------------------------------------------
+// exchange (exchange.cuh) — out-of-line parts that report errors through fail()
+// ------------------------------------------------------------------------------------------------
+namespace blastcf {
+
+int nccl_fail(ncclResult_t r, const char *what) {
+  NcclApi *api = nccl_api();
+  return fail(BLAST_CF_ENCCL, "%s: %s", what, api && api->GetErrorString ? api->GetErrorString(r) : "NCCL error");
+}
+
+#define NCCL_TRY(expr, what)                       \
+  do {                                             \
+    ncclResult_t r_ = (expr);                      \
+    if (r_ != ncclSuccess) return nccl_fail(r_, what); \
+  } while (0)
+
+int nccl_get_unique_id(void *out) {
+  NcclApi *api = nccl_api();
+  if (!api) return fail(BLAST_CF_ENCCL, "cannot dlopen NCCL (set BLAST_CF_NCCL_LIB)");
+  NCCL_TRY(api->GetUniqueId((ncclUniqueId *)out), "ncclGetUniqueId");
+  return BLAST_CF_OK;
+}
+
+int exchange_create(Exchange **out, const blast_cf_mesh *mesh, int dim, int64_t nn, cudaStream_t stream,
+                    const void *uid) {
+  *out = nullptr;
+  NcclApi *api = nccl_api();
+  if (!api) return fail(BLAST_CF_ENCCL, "cannot dlopen NCCL (set BLAST_CF_NCCL_LIB)");
+  if (mesh->num_neighbors < 0 || (mesh->num_neighbors > 0 && (!mesh->nbr_rank || !mesh->nbr_offset || !mesh->nbr_nodes)))
+    return fail(BLAST_CF_EINVAL, "neighbour lists");
+  for (int i = 0; i < mesh->num_neighbors; ++i) {
+    if (mesh->nbr_rank[i] < 0 || mesh->nbr_rank[i] >= mesh->nranks || mesh->nbr_rank[i] == mesh->rank ||
+        (i > 0 && mesh->nbr_rank[i] <= mesh->nbr_rank[i - 1]) || mesh->nbr_offset[i + 1] < mesh->nbr_offset[i])
+      return fail(BLAST_CF_EINVAL, "neighbour %d: ranks must be ascending, distinct from own rank", i);
+  }
+  const int64_t total = mesh->num_neighbors > 0 ? mesh->nbr_offset[mesh->num_neighbors] : 0;
+  for (int64_t r = 0; r < total; ++r)
+    if (mesh->nbr_nodes[r] < 0 || mesh->nbr_nodes[r] >= nn) return fail(BLAST_CF_EINVAL, "nbr_nodes[%lld]", (long long)r);
+  Exchange *x = new (std::nothrow) Exchange();
+  if (!x) return fail(BLAST_CF_ENOMEM, "host allocation");
+  x->api = api; x->rank = mesh->rank; x->nranks = mesh->nranks; x->dim = dim; x->nn = nn;
+  x->num_nbr = mesh->num_neighbors; x->stream = stream; x->nrows = total;
+  x->nbr_rank.assign(mesh->nbr_rank, mesh->nbr_rank + x->num_nbr);
+  x->nbr_offset.assign(mesh->nbr_offset, mesh->nbr_offset + x->num_nbr + 1);
+  ExchangePlan pl = build_plan(x->rank, x->num_nbr, mesh->nbr_rank, mesh->nbr_offset, mesh->nbr_nodes);
+  x->nu = (int64_t)pl.unique_nodes.size();
+  int rc;
+  if ((rc = upload(&x->d_rows, mesh->nbr_nodes, (size_t)total)) ||
+      (rc = upload(&x->d_unodes, pl.unique_nodes.data(), pl.unique_nodes.size())) ||
+      (rc = upload(&x->d_sptr, pl.src_ptr.data(), pl.src_ptr.size())) ||
+      (rc = upload(&x->d_src, pl.src.data(), pl.src.size()))) {
+    exchange_destroy(x);
+    return rc;
+  }
+  if (cudaMalloc(&x->d_send, std::max<int64_t>(total * dim, 1) * sizeof(double)) != cudaSuccess ||
+      cudaMalloc(&x->d_recv, std::max<int64_t>(total * dim, 1) * sizeof(double)) != cudaSuccess ||
+      cudaMalloc(&x->d_tmp, 2 * sizeof(double)) != cudaSuccess) {
+    exchange_destroy(x);
+    return fail(BLAST_CF_ENOMEM, "exchange buffers");
+  }
+  ncclUniqueId id;
+  memcpy(&id, uid, sizeof id);
+  ncclResult_t r = api->CommInitRank(&x->comm, x->nranks, id, x->rank);
+  if (r != ncclSuccess) {
+    x->comm = nullptr;
+    exchange_destroy(x);
+    return nccl_fail(r, "ncclCommInitRank");
+  }
+  *out = x;
+  return BLAST_CF_OK;
+}
+
+int exchange_allreduce_sum2(Exchange *x, double *a, double *b) {
+  double hv[2] = {*a, *b};
+  CUDA_TRY(cudaMemcpy(x->d_tmp, hv, sizeof hv, cudaMemcpyHostToDevice));
+  NCCL_TRY(x->api->AllReduce(x->d_tmp, x->d_tmp, 2, ncclDouble, ncclSum, x->comm, x->stream), "ncclAllReduce(sum)");
+  CUDA_TRY(cudaStreamSynchronize(x->stream));
+  CUDA_TRY(cudaMemcpy(hv, x->d_tmp, sizeof hv, cudaMemcpyDeviceToHost));
+  *a = hv[0];
+  *b = hv[1];
+  return BLAST_CF_OK;
+}
+
+int exchange_run(Exchange *x, double *F1, double *dt) {
+  const int dim = x->dim;
+  if (x->nrows > 0) {
+    const int blocks = (int)std::min<int64_t>((x->nrows + 255) / 256, 1184);
+    xch_pack<<<blocks, 256, 0, x->stream>>>(F1, x->nn, dim, x->d_rows, x->nrows, x->d_send);
+  }
+  NCCL_TRY(x->api->GroupStart(), "ncclGroupStart");
+  for (int i = 0; i < x->num_nbr; ++i) {
+    const int64_t o = x->nbr_offset[i], cnt = x->nbr_offset[i + 1] - o;
+    if (cnt == 0) continue;
+    NCCL_TRY(x->api->Send(x->d_send + o * dim, (size_t)cnt * dim, ncclDouble, x->nbr_rank[i], x->comm, x->stream), "ncclSend");
+    NCCL_TRY(x->api->Recv(x->d_recv + o * dim, (size_t)cnt * dim, ncclDouble, x->nbr_rank[i], x->comm, x->stream), "ncclRecv");
+  }
+  NCCL_TRY(x->api->GroupEnd(), "ncclGroupEnd");
+  NCCL_TRY(x->api->AllReduce(dt, dt, 1, ncclDouble, ncclMin, x->comm, x->stream), "ncclAllReduce(min dt)");
+  if (x->nu > 0) {
+    const int blocks = (int)std::min<int64_t>((x->nu + 255) / 256, 1184);
+    xch_combine<<<blocks, 256, 0, x->stream>>>(F1, x->nn, dim, x->d_unodes, x->nu, x->d_sptr, x->d_src, x->d_send,
+                                               x->d_recv);
+  }
+  return BLAST_CF_OK;
+}
+
+}  // namespace blastcf
+
+struct blast_cf {
+  int dim = 0, k = 0, nk = 0, nt = 0, nq = 0;
+  int64_t Z = 0, nn = 0;
+  blast_cf_params params{};
+  double h0 = 0.0;
+  cudaStream_t stream = nullptr;
+  int device = 0;
+  KB1Variant var{};
+  int ncta = 0, regs = 0, local_bytes = 0;
+  // device memory
+  double *d_tab = nullptr, *d_J0inv = nullptr, *d_gamma = nullptr, *d_Fz1 = nullptr, *d_ctadt = nullptr;
+  int32_t *d_zone_nodes = nullptr, *d_ptr = nullptr, *d_ent = nullptr;
+  // host-eval staging
+  double *d_in = nullptr, *d_out = nullptr;
+  // timing
+  bool timing = false;
+  cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+  // multi-GPU
+  blastcf::Exchange *xch = nullptr;
+};
+
+namespace {
+
+void free_handle(blast_cf *h) {
+  if (!h) return;
+  cudaFree(h->d_tab); cudaFree(h->d_J0inv); cudaFree(h->d_gamma); cudaFree(h->d_Fz1); cudaFree(h->d_ctadt);
+  cudaFree(h->d_zone_nodes); cudaFree(h->d_ptr); cudaFree(h->d_ent); cudaFree(h->d_in); cudaFree(h->d_out);
+  for (auto &e : h->ev)
+    if (e) cudaEventDestroy(e);
+  if (h->xch) blastcf::exchange_destroy(h->xch);
+  delete h;
+}
+
+
+int check_async(blast_cf *h) {
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(BLAST_CF_ECUDA, "CUDA error: %s", cudaGetErrorString(e));
+  (void)h;
+  return BLAST_CF_OK;
+}
+
+double flops_per_zone(int dim, int k) {
+  // sum-factorized contractions + counted pointwise flops (FMA = 2 flops; each
+  // div / sqrt / rsqrt / acos / cos = 1 flop).
+  const double n = 2 * k, p = k + 1, t = k;
+  if (dim == 3) {
+    const double contr = 9.0 * (4 * n * p * p * p + 6 * n * n * p * p + 6 * n * n * n * p) +
+                         4.0 * (n * t * t * t + n * n * t * t + n * n * n * t) + 2.0 * 9 * n * n * n;
+    return contr + 420.0 * n * n * n;
+  }
+  const double contr = 6.0 * (4 * n * p * p + 4 * n * n * p) + 4.0 * (n * t * t + n * n * t) + 2.0 * 4 * n * n;
+  return contr + 160.0 * n * n;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *blast_cf_last_error(void) { return g_last_error.c_str(); }
+
+const char *blast_cf_error_string(int code) {
+  switch (code) {
+    case BLAST_CF_OK: return "BLAST_CF_OK";
+    case BLAST_CF_EINVAL: return "BLAST_CF_EINVAL: invalid argument";
+    case BLAST_CF_EUNSUPPORTED: return "BLAST_CF_EUNSUPPORTED: unsupported configuration";
+    case BLAST_CF_ENOMEM: return "BLAST_CF_ENOMEM: out of memory";
+    case BLAST_CF_ECUDA: return "BLAST_CF_ECUDA: CUDA error";
+    case BLAST_CF_ENCCL: return "BLAST_CF_ENCCL: NCCL error";
+  }
+  return "BLAST_CF_E?: unknown error code";
+}
+
+void blast_cf_default_params(blast_cf_params *p) {
+  if (!p) return;
+  p->cfl = 0.5;
+  p->q_quad = 2.0;
+  p->q_lin = 0.5;
+  p->eps_switch = 1e-12;
+  p->h0 = 0.0;
+  p->use_viscosity = 1;
+  p->use_vorticity = 1;
+}
+
+int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_cf_params *params,
+                    void *cuda_stream, const void *nccl_unique_id, blast_cf **out) {
+  if (!out) return fail(BLAST_CF_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (!mesh) return fail(BLAST_CF_EINVAL, "mesh is NULL");
+  if (mesh->dim != dim || mesh->order != order)
+    return fail(BLAST_CF_EINVAL, "mesh dim/order (%d,%d) != arguments (%d,%d)", mesh->dim, mesh->order, dim, order);
+  if (dim != 2 && dim != 3) return fail(BLAST_CF_EUNSUPPORTED, "dim %d not in {2,3}", dim);
+  if (order < 1 || order > 8) return fail(BLAST_CF_EUNSUPPORTED, "order %d not in [1,8]", order);
+  if (mesh->num_zones < 0 || mesh->num_nodes < 0) return fail(BLAST_CF_EINVAL, "negative sizes");
+  if (mesh->num_zones > 0 && (!mesh->zone_nodes || !mesh->x0)) return fail(BLAST_CF_EINVAL, "zone_nodes/x0 NULL");
+  if (!mesh->mat_gamma || mesh->num_mats < 1) return fail(BLAST_CF_EINVAL, "mat_gamma/num_mats");
+  const int nranks = mesh->nranks < 1 ? 1 : mesh->nranks;
+  if (nranks > 1 && !nccl_unique_id) return fail(BLAST_CF_EINVAL, "nranks > 1 needs nccl_unique_id");
+
+  blast_cf *h = new (std::nothrow) blast_cf();
+  if (!h) return fail(BLAST_CF_ENOMEM, "host allocation");
+  h->dim = dim; h->k = order;
+  int nk = 1, nt = 1, nq = 1;
+  for (int i = 0; i < dim; ++i) { nk *= order + 1; nt *= order; nq *= 2 * order; }
+  h->nk = nk; h->nt = nt; h->nq = nq;
+  h->Z = mesh->num_zones; h->nn = mesh->num_nodes;
+  if (params) h->params = *params; else blast_cf_default_params(&h->params);
+  h->stream = (cudaStream_t)cuda_stream;
+  int rc = BLAST_CF_OK;
+  auto bail = [&](int code) { free_handle(h); return code; };
+  if (cudaGetDevice(&h->device) != cudaSuccess) return bail(fail(BLAST_CF_ECUDA, "no CUDA device"));
+
+  // ---- validate the map ----
+  const int64_t Z = h->Z, nn = h->nn;
+  for (int64_t i = 0; i < Z * nk; ++i) {
+    const int32_t nd = mesh->zone_nodes[i];
+    if (nd < 0 || nd >= nn) return bail(fail(BLAST_CF_EINVAL, "zone_nodes[%lld] = %d out of range", (long long)i, nd));
+  }
+  std::vector<double> zgam(Z);
+  for (int64_t z = 0; z < Z; ++z) {
+    const int m = mesh->zone_mat ? mesh->zone_mat[z] : 0;
+    if (m < 0 || m >= mesh->num_mats) return bail(fail(BLAST_CF_EINVAL, "zone_mat[%lld] = %d", (long long)z, m));
+    zgam[z] = mesh->mat_gamma[m];
+  }
+
+  // ---- tables ----
+  const blastcf::Tables1D T = blastcf::build_tables(order);
+  const int n = T.n, p = T.p, t = T.t;
+  std::vector<double> tab;
+  tab.insert(tab.end(), T.B.begin(), T.B.end());
+  tab.insert(tab.end(), T.G.begin(), T.G.end());
+  tab.insert(tab.end(), T.Phi.begin(), T.Phi.end());
+  tab.insert(tab.end(), T.qwt.begin(), T.qwt.end());
+
+  // ---- per-zone J0^{-1} of the affine initial zones and the volume ----
+  std::vector<double> J0inv((size_t)Z * dim * dim);
+  long double vol = 0.0L;
+  bool affine = true;
+  int64_t bad_zone = -1;
+  for (int64_t z = 0; z < Z; ++z) {
+    const int32_t *zn = mesh->zone_nodes + z * nk;
+    long double J[3][3] = {{0}}, X0[3];
+    for (int c = 0; c < dim; ++c) X0[c] = mesh->x0[c * nn + zn[0]];
+    for (int d = 0; d < dim; ++d) {
+      int a = (d == 0 ? order : d == 1 ? order * p : order * p * p);   // vertex with l_d = k
+      for (int c = 0; c < dim; ++c) J[c][d] = (long double)mesh->x0[c * nn + zn[a]] - X0[c];
+    }
+    // affinity: x_a = x_0 + J xi_a for every node a
+    long double scale = 0.0L;
+    for (int c = 0; c < dim; ++c)
+      for (int d = 0; d < dim; ++d) scale = std::max(scale, fabsl(J[c][d]));
+    for (int a = 0; a < nk && affine; ++a) {
+      const int li[3] = {a % p, (a / p) % p, a / (p * p)};
+      for (int c = 0; c < dim; ++c) {
+        long double xa = X0[c];
+        for (int d = 0; d < dim; ++d) xa += J[c][d] * (long double)T.gll[li[d]];
+        if (fabsl(xa - (long double)mesh->x0[c * nn + zn[a]]) > 1e-11L * scale) { affine = false; bad_zone = z; }
+      }
+    }
+    long double det, inv[3][3];
+    if (dim == 2) {
+      det = J[0][0] * J[1][1] - J[0][1] * J[1][0];
+      inv[0][0] = J[1][1] / det; inv[0][1] = -J[0][1] / det;
+      inv[1][0] = -J[1][0] / det; inv[1][1] = J[0][0] / det;
+    } else {
+      const long double c00 = J[1][1] * J[2][2] - J[1][2] * J[2][1], c01 = J[0][2] * J[2][1] - J[0][1] * J[2][2],
+                        c02 = J[0][1] * J[1][2] - J[0][2] * J[1][1], c10 = J[1][2] * J[2][0] - J[1][0] * J[2][2],
+                        c11 = J[0][0] * J[2][2] - J[0][2] * J[2][0], c12 = J[0][2] * J[1][0] - J[0][0] * J[1][2],
+                        c20 = J[1][0] * J[2][1] - J[1][1] * J[2][0], c21 = J[0][1] * J[2][0] - J[0][0] * J[2][1],
+                        c22 = J[0][0] * J[1][1] - J[0][1] * J[1][0];
+      det = J[0][0] * c00 + J[0][1] * c10 + J[0][2] * c20;
+      inv[0][0] = c00 / det; inv[0][1] = c01 / det; inv[0][2] = c02 / det;
+      inv[1][0] = c10 / det; inv[1][1] = c11 / det; inv[1][2] = c12 / det;
+      inv[2][0] = c20 / det; inv[2][1] = c21 / det; inv[2][2] = c22 / det;
+    }
+    vol += det;
+    for (int c = 0; c < dim; ++c)
+      for (int d = 0; d < dim; ++d) J0inv[(size_t)z * dim * dim + c * dim + d] = (double)inv[c][d];
+  }
+  if (!affine && h->params.use_viscosity)
+    return bail(fail(BLAST_CF_EUNSUPPORTED,
+                     "initial zone %lld is not affine: the viscosity length scale needs per-point J0 (not built)",
+                     (long long)bad_zone));
+
+  // ---- multi-GPU: communicator, global volume / zone count for h0 ----
+  double gvol = (double)vol, gz = (double)Z;
+  if (nranks > 1) {
+    rc = blastcf::exchange_create(&h->xch, mesh, dim, nn, h->stream, nccl_unique_id);
+    if (rc) { free_handle(h); return rc; }
+    rc = blastcf::exchange_allreduce_sum2(h->xch, &gvol, &gz);
+    if (rc) { free_handle(h); return rc; }
+  }
+  h->h0 = h->params.h0 > 0.0 ? h->params.h0 : pow(gvol / gz, 1.0 / dim) / order;
+
+  // ---- inverse map: node -> entries z*dim*nk + a in ascending zone id ----
+  std::vector<int32_t> ptr(nn + 1, 0), ent((size_t)Z * nk);
+  if ((double)Z * dim * nk >= 2147483647.0) return bail(fail(BLAST_CF_EUNSUPPORTED, "too many zones for int32 entries"));
+  for (int64_t i = 0; i < Z * nk; ++i) ptr[mesh->zone_nodes[i] + 1]++;
+  for (int64_t i = 0; i < nn; ++i) ptr[i + 1] += ptr[i];
+  {
+    std::vector<int32_t> fill(ptr.begin(), ptr.end() - 1);
+    for (int64_t z = 0; z < Z; ++z)
+      for (int a = 0; a < nk; ++a) ent[fill[mesh->zone_nodes[z * nk + a]]++] = (int32_t)(z * dim * nk + a);
+  }
+
+  // ---- kernel variant ----
+  h->var = select_variant(dim, order);
+  if (!h->var.launch) return bail(fail(BLAST_CF_EUNSUPPORTED, "no kernel for dim %d order %d", dim, order));
+  if (cudaFuncSetAttribute(h->var.func, cudaFuncAttributeMaxDynamicSharedMemorySize, h->var.smem) != cudaSuccess)
+    return bail(fail(BLAST_CF_ECUDA, "cudaFuncSetAttribute(smem=%d): %s", h->var.smem,
+                     cudaGetErrorString(cudaGetLastError())));
+  cudaFuncAttributes fa;
+  if (cudaFuncGetAttributes(&fa, h->var.func) == cudaSuccess) {
+    h->regs = fa.numRegs;
+    h->local_bytes = (int)fa.localSizeBytes;
+  }
+  h->ncta = (int)((Z + h->var.zpc - 1) / h->var.zpc);
+
+  // ---- uploads ----
+  if ((rc = upload(&h->d_tab, tab.data(), tab.size())) ||
+      (rc = upload(&h->d_J0inv, J0inv.data(), J0inv.size())) ||
+      (rc = upload(&h->d_gamma, zgam.data(), zgam.size())) ||
+      (rc = upload(&h->d_zone_nodes, mesh->zone_nodes, (size_t)Z * nk)) ||
+      (rc = upload(&h->d_ptr, ptr.data(), ptr.size())) || (rc = upload(&h->d_ent, ent.data(), ent.size())))
+    return bail(rc);
+  if (cudaMalloc(&h->d_Fz1, std::max<size_t>((size_t)Z * dim * nk, 1) * sizeof(double)) != cudaSuccess ||
+      cudaMalloc(&h->d_ctadt, std::max(h->ncta, 1) * sizeof(double)) != cudaSuccess)
+    return bail(fail(BLAST_CF_ENOMEM, "workspace allocation"));
+  for (auto &e : h->ev)
+    if (cudaEventCreate(&e) != cudaSuccess) return bail(fail(BLAST_CF_ECUDA, "event create"));
+  *out = h;
+  return BLAST_CF_OK;
+}
+
+static int eval_impl(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                     double *out_Fdot1, double *out_FTv, double *out_dt_min, double *Sq) {
+  if (!h) return fail(BLAST_CF_EINVAL, "handle is NULL");
+  if (!out_dt_min || ((!x || !v || !out_Fdot1) && h->nn > 0) || ((!e || !rho0detJ0 || !out_FTv) && h->Z > 0))
+    return fail(BLAST_CF_EINVAL, "NULL array argument");
+  int rc = check_async(h);
+  if (rc) return rc;
+  KB1Args a;
+  a.x = x; a.v = v; a.e = e; a.rho0detJ0 = rho0detJ0;
+  a.zone_nodes = h->d_zone_nodes; a.J0inv = h->d_J0inv; a.zone_gamma = h->d_gamma; a.tab = h->d_tab;
+  a.Fz1 = h->d_Fz1; a.FTv = out_FTv; a.cta_dt = h->d_ctadt; a.Sq = Sq;
+  a.num_zones = h->Z; a.num_nodes = h->nn;
+  a.ph.cfl = h->params.cfl; a.ph.q_quad = h->params.q_quad; a.ph.q_lin = h->params.q_lin;
+  a.ph.eps_sw = h->params.eps_switch; a.ph.h0 = h->h0; a.ph.inv_k = 1.0 / h->k;
+  a.ph.use_visc = h->params.use_viscosity; a.ph.use_vort = h->params.use_vorticity;
+  if (h->timing) cudaEventRecord(h->ev[0], h->stream);
+  if (h->ncta > 0) h->var.launch(a, h->ncta, h->stream);
+  if (h->timing) cudaEventRecord(h->ev[1], h->stream);
+  const int gthreads = 256;
+  int64_t gblocks = (h->nn + gthreads - 1) / gthreads;
+  gblocks = std::max<int64_t>(1, std::min<int64_t>(gblocks, 148 * 16));
+  kb2_gather<<<(int)gblocks, gthreads, 0, h->stream>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->dim, h->nk, out_Fdot1,
+                                                        h->d_ctadt, h->ncta, out_dt_min);
+  if (h->timing) cudaEventRecord(h->ev[2], h->stream);
+  if (h->xch) {
+    rc = blastcf::exchange_run(h->xch, out_Fdot1, out_dt_min);
+    if (rc) return rc;
+  }
+  if (h->timing) cudaEventRecord(h->ev[3], h->stream);
+  return check_async(h);
+}
+
+int blast_cf_eval(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                  double *out_Fdot1, double *out_FTv, double *out_dt_min) {
+  return eval_impl(h, x, v, e, rho0detJ0, out_Fdot1, out_FTv, out_dt_min, nullptr);
+}
+
+int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                       double *out_Fdot1, double *out_FTv, double *out_dt_min) {
+  if (!h) return fail(BLAST_CF_EINVAL, "handle is NULL");
+  const size_t nx = (size_t)h->dim * h->nn, ne = (size_t)h->Z * h->nt, nr = (size_t)h->Z * h->nq;
+  if (!h->d_in) {
+    CUDA_TRY(cudaMalloc(&h->d_in, (2 * nx + ne + nr + 1) * sizeof(double)));
+    CUDA_TRY(cudaMalloc(&h->d_out, (nx + ne + 1) * sizeof(double)));
+  }
+  double *dx = h->d_in, *dv = dx + nx, *de = dv + nx, *dr = de + ne;
+  double *dF = h->d_out, *dT = dF + nx, *dd = dT + ne;
+  CUDA_TRY(cudaMemcpyAsync(dx, x, nx * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(dv, v, nx * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(de, e, ne * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(dr, rho0detJ0, nr * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+  int rc = blast_cf_eval(h, dx, dv, de, dr, dF, dT, dd);
+  if (rc) return rc;
+  CUDA_TRY(cudaMemcpyAsync(out_Fdot1, dF, nx * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(out_FTv, dT, ne * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaMemcpyAsync(out_dt_min, dd, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  return BLAST_CF_OK;
+}
+
+int blast_cf_eval_debug_Fz(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                           double *out_Fz) {
+  if (!h || !out_Fz) return fail(BLAST_CF_EINVAL, "NULL argument");
+  const size_t nx = (size_t)h->dim * h->nn, ne = (size_t)h->Z * h->nt;
+  double *Sq = nullptr, *F1 = nullptr, *FT = nullptr;
+  CUDA_TRY(cudaMalloc(&Sq, std::max<size_t>((size_t)h->Z * h->nq * h->dim * h->dim, 1) * sizeof(double)));
+  CUDA_TRY(cudaMalloc(&F1, (nx + 1) * sizeof(double)));
+  CUDA_TRY(cudaMalloc(&FT, (ne + 2) * sizeof(double)));
+  int rc = eval_impl(h, x, v, e, rho0detJ0, F1, FT, FT + ne, Sq);
+  if (!rc && h->Z > 0) {
+    if (h->dim == 3) kbd_form_Fz<3><<<(int)h->Z, 128, 0, h->stream>>>(Sq, h->d_tab, h->k, h->Z, out_Fz);
+    else kbd_form_Fz<2><<<(int)h->Z, 128, 0, h->stream>>>(Sq, h->d_tab, h->k, h->Z, out_Fz);
+    if (cudaStreamSynchronize(h->stream) != cudaSuccess) rc = fail(BLAST_CF_ECUDA, "debug F_z kernel");
+  }
+  cudaFree(Sq); cudaFree(F1); cudaFree(FT);
+  return rc;
+}
+
+int blast_cf_get_info(const blast_cf *h, blast_cf_info *info) {
+  if (!h || !info) return fail(BLAST_CF_EINVAL, "NULL argument");
+  info->dim = h->dim; info->order = h->k; info->nq = h->nq; info->nk = h->nk; info->nt = h->nt;
+  info->num_zones = h->Z; info->num_nodes = h->nn; info->h0 = h->h0;
+  info->zones_per_cta = h->var.zpc; info->threads_per_cta = h->var.nth; info->num_ctas = h->ncta;
+  info->smem_bytes = h->var.smem; info->regs_per_thread = h->regs; info->local_bytes = h->local_bytes;
+  info->flops_per_zone = flops_per_zone(h->dim, h->k);
+  // x, v read once, F.1 written once, e read, F^T v written, rho0|J0| read, dt
+  info->alg_bytes = 8.0 * (3.0 * h->dim * h->nn + (double)h->Z * (2.0 * h->nt + h->nq)) + 8.0;
+  info->kernels_per_eval = 2 + (h->xch ? blastcf::exchange_kernels(h->xch) : 0);
+  return BLAST_CF_OK;
+}
+
+int blast_cf_set_timing(blast_cf *h, int enable) {
+  if (!h) return fail(BLAST_CF_EINVAL, "handle is NULL");
+  h->timing = enable != 0;
+  return BLAST_CF_OK;
+}
+
+int blast_cf_kernel_times(blast_cf *h, float *ms3) {
+  if (!h || !ms3) return fail(BLAST_CF_EINVAL, "NULL argument");
+  if (!h->timing) return fail(BLAST_CF_EINVAL, "timing not enabled");
+  CUDA_TRY(cudaEventSynchronize(h->ev[3]));
+  CUDA_TRY(cudaEventElapsedTime(&ms3[0], h->ev[0], h->ev[1]));
+  CUDA_TRY(cudaEventElapsedTime(&ms3[1], h->ev[1], h->ev[2]));
+  CUDA_TRY(cudaEventElapsedTime(&ms3[2], h->ev[2], h->ev[3]));
+  return BLAST_CF_OK;
+}
+
+int blast_cf_debug_cta_dt(blast_cf *h, double *host_out, int64_t capacity, int32_t *num_ctas, int32_t *zones_per_cta) {
+  if (!h || !num_ctas || !zones_per_cta) return fail(BLAST_CF_EINVAL, "NULL argument");
+  *num_ctas = h->ncta;
+  *zones_per_cta = h->var.zpc;
+  if (host_out && h->ncta > 0) {
+    if (capacity < h->ncta) return fail(BLAST_CF_EINVAL, "capacity %lld < %d", (long long)capacity, h->ncta);
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    CUDA_TRY(cudaMemcpy(host_out, h->d_ctadt, h->ncta * sizeof(double), cudaMemcpyDeviceToHost));
+  }
+  return BLAST_CF_OK;
+}
+
+int blast_cf_destroy(blast_cf *h) {
+  if (!h) return fail(BLAST_CF_EINVAL, "handle is NULL");
+  if (h->stream) cudaStreamSynchronize(h->stream);
+  else cudaDeviceSynchronize();
+  free_handle(h);
+  return BLAST_CF_OK;
+}
+
+int blast_cf_exchange_plan(int32_t rank, int32_t num_neighbors, const int32_t *nbr_rank, const int64_t *nbr_offset,
+                           const int32_t *nbr_nodes, int64_t capacity, int64_t *num_unique, int32_t *unique_nodes,
+                           int64_t *src_ptr, int64_t *src) {
+  if (num_neighbors < 0 || !num_unique || (num_neighbors > 0 && (!nbr_rank || !nbr_offset || !nbr_nodes)))
+    return fail(BLAST_CF_EINVAL, "NULL argument");
+  blastcf::ExchangePlan pl = blastcf::build_plan(rank, num_neighbors, nbr_rank, nbr_offset, nbr_nodes);
+  *num_unique = (int64_t)pl.unique_nodes.size();
+  if ((int64_t)pl.src.size() > capacity || (int64_t)pl.src_ptr.size() > capacity + 1)
+    return fail(BLAST_CF_EINVAL, "capacity %lld too small", (long long)capacity);
+  std::copy(pl.unique_nodes.begin(), pl.unique_nodes.end(), unique_nodes);
+  std::copy(pl.src_ptr.begin(), pl.src_ptr.end(), src_ptr);
+  std::copy(pl.src.begin(), pl.src.end(), src);
+  return BLAST_CF_OK;
+}
+
+int blast_cf_nccl_unique_id_size(void) { return blastcf::nccl_unique_id_bytes(); }
+
+int blast_cf_nccl_get_unique_id(void *out) {
+  if (!out) return fail(BLAST_CF_EINVAL, "NULL argument");
+  return blastcf::nccl_get_unique_id(out);
+}
+
+}  // extern "C"

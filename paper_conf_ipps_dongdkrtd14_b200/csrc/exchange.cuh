@@ -1,0 +1,170 @@
+// Multi-GPU shared-DOF exchange (§3.4).
+//
+// BLAST/MFEM assemble zone contributions across MPI tasks through groups of shared DOFs with a master
+// per group, and reduce the minimum time step with MPI.  Here: one process per B200,
+// NCCL over NVLink.  After KB2 every rank holds its partial F.1 on the nodes it shares; it
+//   1. packs them per neighbour (rows ordered by global node id, identical on both sides),
+//   2. exchanges them with grouped ncclSend / ncclRecv on the handle's stream,
+//   3. sums, for every shared node, the partials of all sharing ranks in ASCENDING RANK order, so every
+//      sharer ends with bitwise identical values (reading R20),
+// and takes the global min dt with ncclAllReduce(min).
+// NCCL is loaded with dlopen at create time so that single-GPU use never touches it.
+#pragma once
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <cstdint>
+#include <cstdlib>
+#include <vector>
+
+#include "nccl.h"
+
+namespace blastcf {
+
+struct NcclApi {
+  void *lib = nullptr;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId *) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*GroupStart)() = nullptr;
+  ncclResult_t (*GroupEnd)() = nullptr;
+  ncclResult_t (*Send)(const void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Recv)(void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*AllReduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                            cudaStream_t) = nullptr;
+  const char *(*GetErrorString)(ncclResult_t) = nullptr;
+};
+
+inline NcclApi *nccl_api() {
+  static NcclApi api;
+  static bool tried = false;
+  if (tried) return api.lib ? &api : nullptr;
+  tried = true;
+  const char *cands[3] = {getenv("BLAST_CF_NCCL_LIB"), "libnccl.so.2", "libnccl.so"};
+  for (const char *c : cands) {
+    if (!c || !*c) continue;
+    api.lib = dlopen(c, RTLD_NOW | RTLD_GLOBAL);
+    if (api.lib) break;
+  }
+  if (!api.lib) return nullptr;
+#define LOADSYM(field, name) api.field = (decltype(api.field))dlsym(api.lib, name)
+  LOADSYM(GetUniqueId, "ncclGetUniqueId");
+  LOADSYM(CommInitRank, "ncclCommInitRank");
+  LOADSYM(CommDestroy, "ncclCommDestroy");
+  LOADSYM(GroupStart, "ncclGroupStart");
+  LOADSYM(GroupEnd, "ncclGroupEnd");
+  LOADSYM(Send, "ncclSend");
+  LOADSYM(Recv, "ncclRecv");
+  LOADSYM(AllReduce, "ncclAllReduce");
+  LOADSYM(GetErrorString, "ncclGetErrorString");
+#undef LOADSYM
+  if (!api.GetUniqueId || !api.CommInitRank || !api.Send || !api.Recv || !api.AllReduce || !api.GroupStart ||
+      !api.GroupEnd || !api.CommDestroy) {
+    api.lib = nullptr;
+    return nullptr;
+  }
+  return &api;
+}
+
+inline int nccl_unique_id_bytes() { return (int)sizeof(ncclUniqueId); }
+
+int nccl_fail(ncclResult_t r, const char *what);
+
+// ---------------------------------------------------------------------------------------------
+// Host plan (no CUDA): rows of the pack buffers and the ordered source list of every shared node.
+// Row r of the send (and recv) buffer holds the dim partials of nbr_nodes[r] for neighbour i with
+// nbr_offset[i] <= r < nbr_offset[i+1].  For each unique shared node u (ascending local id):
+// sources src[src_ptr[u] .. src_ptr[u+1]) in ascending rank; src >= 0: own partial in send row src,
+// src < 0: neighbour partial in recv row (-src - 1).
+// ---------------------------------------------------------------------------------------------
+struct ExchangePlan {
+  std::vector<int32_t> unique_nodes;
+  std::vector<int64_t> src_ptr, src;
+};
+
+inline ExchangePlan build_plan(int rank, int num_nbr, const int32_t *nbr_rank, const int64_t *nbr_offset,
+                               const int32_t *nbr_nodes) {
+  ExchangePlan pl;
+  const int64_t total = num_nbr > 0 ? nbr_offset[num_nbr] : 0;
+  // (node, rank, row) triples
+  struct E { int32_t node, rank; int64_t row; };
+  std::vector<E> es;
+  es.reserve(total);
+  for (int i = 0; i < num_nbr; ++i)
+    for (int64_t r = nbr_offset[i]; r < nbr_offset[i + 1]; ++r) es.push_back({nbr_nodes[r], nbr_rank[i], r});
+  std::sort(es.begin(), es.end(), [](const E &a, const E &b) {
+    return a.node != b.node ? a.node < b.node : a.rank < b.rank;
+  });
+  pl.src_ptr.push_back(0);
+  for (size_t i = 0; i < es.size();) {
+    size_t j = i;
+    while (j < es.size() && es[j].node == es[i].node) ++j;
+    pl.unique_nodes.push_back(es[i].node);
+    bool own_done = false;
+    for (size_t t = i; t < j; ++t) {
+      if (!own_done && rank < es[t].rank) { pl.src.push_back(es[i].row); own_done = true; }
+      pl.src.push_back(-es[t].row - 1);
+    }
+    if (!own_done) pl.src.push_back(es[i].row);
+    pl.src_ptr.push_back((int64_t)pl.src.size());
+    i = j;
+  }
+  return pl;
+}
+
+// ---------------------------------------------------------------------------------------------
+// device side
+// ---------------------------------------------------------------------------------------------
+__global__ void xch_pack(const double *__restrict__ F1, int64_t nn, int dim, const int32_t *__restrict__ rows,
+                         int64_t nrows, double *__restrict__ send) {
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < nrows; r += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t node = rows[r];
+    for (int c = 0; c < dim; ++c) send[r * dim + c] = F1[c * nn + node];
+  }
+}
+
+__global__ void xch_combine(double *__restrict__ F1, int64_t nn, int dim, const int32_t *__restrict__ unodes,
+                            int64_t nu, const int64_t *__restrict__ sptr, const int64_t *__restrict__ src,
+                            const double *__restrict__ send, const double *__restrict__ recv) {
+  for (int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; u < nu; u += (int64_t)gridDim.x * blockDim.x) {
+    double s[3] = {0.0, 0.0, 0.0};
+    for (int64_t i = sptr[u]; i < sptr[u + 1]; ++i) {
+      const int64_t code = src[i];
+      const double *row = code >= 0 ? send + code * dim : recv + (-code - 1) * dim;
+      for (int c = 0; c < dim; ++c) s[c] += row[c];
+    }
+    const int64_t node = unodes[u];
+    for (int c = 0; c < dim; ++c) F1[c * nn + node] = s[c];
+  }
+}
+
+struct Exchange {
+  NcclApi *api = nullptr;
+  ncclComm_t comm = nullptr;
+  int rank = 0, nranks = 1, dim = 0, num_nbr = 0;
+  int64_t nn = 0, nrows = 0, nu = 0;
+  std::vector<int32_t> nbr_rank;
+  std::vector<int64_t> nbr_offset;
+  cudaStream_t stream = nullptr;
+  int32_t *d_rows = nullptr, *d_unodes = nullptr;
+  int64_t *d_sptr = nullptr, *d_src = nullptr;
+  double *d_send = nullptr, *d_recv = nullptr, *d_tmp = nullptr;
+};
+
+inline void exchange_destroy(Exchange *x) {
+  if (!x) return;
+  if (x->comm && x->api) x->api->CommDestroy(x->comm);
+  cudaFree(x->d_rows); cudaFree(x->d_unodes); cudaFree(x->d_sptr); cudaFree(x->d_src);
+  cudaFree(x->d_send); cudaFree(x->d_recv); cudaFree(x->d_tmp);
+  delete x;
+}
+
+inline int exchange_kernels(const Exchange *x) { return x->nrows > 0 ? 2 : 0; }
+
+int exchange_create(Exchange **out, const blast_cf_mesh *mesh, int dim, int64_t nn, cudaStream_t stream,
+                    const void *uid);
+int exchange_allreduce_sum2(Exchange *x, double *a, double *b);
+int exchange_run(Exchange *x, double *F1, double *dt);
+int nccl_get_unique_id(void *out);
+
+}  // namespace blastcf

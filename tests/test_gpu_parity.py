@@ -1,0 +1,193 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle on the same seeded inputs.
+
+Bar (BASELINE.json north_star): max-norm relative error <= 1e-12 on F.1, F^T v and dt, i.e.
+    err_F1 = max|F1_gpu - F1_orc| / max|F1_orc|   (likewise F^T v),   err_dt = |dt_gpu - dt_orc| / dt_orc.
+Small cases span several CTAs and a ragged last CTA; the BASELINE sizes (C2-C5, in the bench's launch
+configuration) are checked on sampled nodes/zones the oracle evaluates one by one, plus the argmin-CTA
+dt and properties that hold at any size (momentum, energy identity, determinism).
+"""
+import numpy as np
+import pytest
+
+import synth
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-12
+
+
+def _torch():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    return torch
+
+
+def gpu_eval(mesh, st, params=None, reps=1):
+    torch = _torch()
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    h = cf.from_synth(mesh, params)
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    x, v, e, r = t(st.x), t(st.v), t(st.e), t(st.rho0detJ0)
+    outs = []
+    for _ in range(reps):
+        F1, FTv, dt = h.eval(x, v, e, r)
+        torch.cuda.synchronize()
+        outs.append((F1.cpu().numpy(), FTv.cpu().numpy(), float(dt.cpu()[0])))
+    return h, outs
+
+
+def rel(a, b):
+    return float(np.abs(a - b).max() / max(np.abs(b).max(), 1e-300))
+
+
+def check(mesh, st, orc, oparams=None, gparams=None, tol=TOL):
+    h, [(F1, FTv, dt)] = gpu_eval(mesh, st, gparams)
+    r = orc.evaluate(mesh, st, params=oparams)
+    e1, e2 = rel(F1, r.F1), rel(FTv, r.FTv)
+    e3 = abs(dt - r.dt_min) / r.dt_min if np.isfinite(r.dt_min) and r.dt_min > 0 else abs(dt - r.dt_min)
+    assert e1 <= tol and e2 <= tol and e3 <= tol, (e1, e2, e3, r.diag)
+    return h, (F1, FTv, dt), r
+
+
+# ---------------------------------------------------------------------------------------------
+# small cases: every order in 2D and 3D, both states, ragged CTA tails
+# ---------------------------------------------------------------------------------------------
+@pytest.mark.parametrize("k", list(range(1, 9)))
+def test_2d_all_orders(orc, k):
+    m, s = synth.config("C2", "S1", N=(5, 3), k=k)
+    check(m, s, orc)
+
+
+@pytest.mark.parametrize("k", list(range(1, 9)))
+def test_3d_all_orders(orc, k):
+    N = (3, 2, 2) if k <= 4 else (2, 1, 2)
+    m, s = synth.config("C4", "S1", N=N, k=k)
+    check(m, s, orc)
+
+
+@pytest.mark.parametrize("name,N,which", [
+    ("C1", None, "S0"), ("C1", None, "S1"),
+    ("C2", (16, 16), "S1"), ("C2", (16, 16), "S1b"),
+    ("C3", (6, 5, 4), "S0"), ("C3", (6, 5, 4), "S1"),
+    ("C4", (5, 3, 3), "S0"), ("C4", (5, 3, 3), "S1"),
+    ("C5", (4, 2, 2), "S0"), ("C5", (4, 2, 2), "S1"),
+])
+def test_configs_small(orc, name, N, which):
+    m, s = synth.config(name, which, N=N)
+    check(m, s, orc)
+
+
+def test_c1_exact_oracle_case_bitwise_sane(orc):
+    """C1 (BASELINE configs[0]): one evaluation vs the oracle, plus the closed-form Sedov dt."""
+    m, s = synth.config("C1", "S0")
+    h, (F1, FTv, dt), r = check(m, s, orc)
+    assert abs(dt - 0.018559808466140585) < 1e-15
+    assert np.abs(FTv).max() == 0.0
+
+
+@pytest.mark.parametrize("visc,vort", [(0, 0), (1, 0)])
+def test_param_switches(orc, visc, vort):
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    m, s = synth.config("C3", "S1", N=(3, 3, 3))
+    gp = cf.default_params()
+    gp.use_viscosity, gp.use_vorticity = visc, vort
+    op = orc.Params(use_viscosity=visc, use_vorticity=vort)
+    check(m, s, orc, oparams=op, gparams=gp)
+
+
+def test_inverted_zone_gives_dt_zero(orc):
+    m, s = synth.config("C3", "S1", N=(3, 3, 3))
+    x = s.x.copy()
+    a = m.zone_nodes[13]                         # interior zone: pull its centre node far through a face
+    x[0, a[13]] += 5.0 / 3
+    s2 = synth.State(x, s.v, s.e, s.rho0detJ0)
+    h, [(F1, FTv, dt)] = gpu_eval(m, s2)
+    r = orc.evaluate(m, s2)
+    assert r.diag["n_bad"] > 0 and r.dt_min == 0.0
+    assert dt == 0.0
+
+
+def test_single_zone_and_empty(orc):
+    torch = _torch()
+    m, s = synth.config("C4", "S1", N=(1, 1, 1))
+    check(m, s, orc)
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    h = cf.CornerForce(np.zeros((0, 27), np.int32), np.zeros((3, 0)), 2, 3)
+    F1, FTv, dt = h.eval(*(torch.zeros(sh, dtype=torch.float64, device="cuda") for sh in ((3, 0), (3, 0), (0, 8), (0, 64))))
+    torch.cuda.synchronize()
+    assert float(dt.cpu()[0]) == float("inf")
+
+
+def test_determinism_bitwise():
+    m, s = synth.config("C4", "S1", N=(6, 5, 4))
+    h, outs = gpu_eval(m, s, reps=10)
+    for o in outs[1:]:
+        assert np.array_equal(o[0], outs[0][0]) and np.array_equal(o[1], outs[0][1]) and o[2] == outs[0][2]
+
+
+def test_eval_host_matches_device():
+    torch = _torch()
+    m, s = synth.config("C3", "S1", N=(4, 4, 3))
+    h, [(F1, FTv, dt)] = gpu_eval(m, s)
+    hx = [torch.from_numpy(np.ascontiguousarray(a)).pin_memory() for a in (s.x, s.v, s.e, s.rho0detJ0)]
+    o = h.eval_host(*hx)
+    assert np.array_equal(o[0], F1) and np.array_equal(o[1], FTv) and o[2][0] == dt
+
+
+@pytest.mark.parametrize("name,N,k", [("C1", None, None), ("C3", (2, 2, 1), None), ("C2", (2, 2), 3)])
+def test_debug_Fz_matches_oracle_definition_mode(orc, name, N, k):
+    torch = _torch()
+    m, s = synth.config(name, "S1", N=N, k=k)
+    h, _ = gpu_eval(m, s)
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    Fz = h.eval_debug_Fz(t(s.x), t(s.v), t(s.e), t(s.rho0detJ0)).cpu().numpy()
+    r = orc.evaluate(m, s, definition=True)
+    assert rel(Fz, r.Fz) <= TOL
+
+
+def test_gpu_invariants():
+    m, s = synth.config("C4", "S1", N=(6, 6, 6))
+    h, [(F1, FTv, dt)] = gpu_eval(m, s)
+    assert np.abs(F1.sum(1)).max() <= 1e-13 * np.abs(F1).sum()
+    assert abs((s.v * F1).sum() - FTv.sum()) <= 1e-13 * np.abs(s.v).max() * np.abs(F1).sum()
+
+
+# ---------------------------------------------------------------------------------------------
+# BASELINE sizes (the bench's launch configuration): sampled parity
+# ---------------------------------------------------------------------------------------------
+def sampled_parity(orc, name, which, n_nodes=48, n_zones=48, seed=0):
+    m, s = synth.config(name, which)
+    h, [(F1, FTv, dt)] = gpu_eval(m, s)
+    rng = np.random.default_rng(seed)
+    nodes = rng.choice(m.num_nodes, size=n_nodes, replace=False)
+    inc = np.unique(np.nonzero(np.isin(m.zone_nodes, nodes))[0])
+    extra = rng.choice(m.num_zones, size=n_zones, replace=False)
+    # the CTA holding the GPU's minimum dt: its zones must reproduce dt_min exactly
+    cta_dt, zpc = h.debug_cta_dt()
+    cmin = int(np.argmin(cta_dt))
+    assert cta_dt[cmin] == dt
+    arg_zones = np.arange(cmin * zpc, min((cmin + 1) * zpc, m.num_zones))
+    zones = np.unique(np.concatenate([inc, extra, arg_zones]))
+    h0 = (np.prod(m.L) / m.num_zones) ** (1.0 / m.dim) / m.order   # closed form for the uniform box
+    assert abs(h.info["h0"] - h0) <= 1e-14 * h0
+    r = orc.evaluate(m, s, params=orc.Params(h0=h0), zones=zones)
+    scale_F = np.abs(F1).max()
+    assert np.abs(F1[:, nodes] - r.F1[:, nodes]).max() <= TOL * scale_F
+    sub = np.searchsorted(zones, np.arange(m.num_zones))
+    pos = np.searchsorted(zones, zones)
+    assert np.abs(FTv[zones] - r.FTv[pos]).max() <= TOL * np.abs(FTv).max()
+    # per-CTA dt of every sampled zone's CTA must bound the oracle's zone dt, and the argmin CTA matches
+    odt = r.dtz[np.searchsorted(zones, arg_zones)].min()
+    assert abs(dt - odt) <= TOL * odt, (dt, odt)
+    for z, dz in zip(zones, r.dtz):
+        assert cta_dt[z // zpc] <= dz * (1 + TOL)
+    # any-size properties
+    assert np.abs(F1.sum(1)).max() <= 1e-12 * np.abs(F1).sum()
+    assert abs((s.v * F1).sum() - FTv.sum()) <= 1e-12 * np.abs(s.v).max() * np.abs(F1).sum()
+    del sub
+
+
+@pytest.mark.parametrize("name,which", [("C2", "S1"), ("C2", "S1b"), ("C3", "S1"), ("C4", "S1"), ("C4", "S0"),
+                                        ("C5", "S1")])
+def test_full_size_sampled(orc, name, which):
+    sampled_parity(orc, name, which, n_nodes=24 if name == "C5" else 48, n_zones=8 if name == "C5" else 48)
