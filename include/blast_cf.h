@@ -132,8 +132,9 @@ int blast_cf_get_info(const blast_cf *h, blast_cf_info *info);
 int blast_cf_set_timing(blast_cf *h, int enable);
 int blast_cf_kernel_times(blast_cf *h, float *ms3);
 
-/* Tests only: the per-CTA minimum dt of the last eval (CTA c covers zones [c*zpc, (c+1)*zpc)), copied
- * to host_out[capacity] after synchronizing the stream.  host_out NULL: only report the sizes. */
+/* Tests only: the per-CTA minimum dt of the last eval, copied to host_out[capacity] after synchronizing
+ * the stream (host_out NULL: only report the sizes).  Zone z belongs to CTA (z / zones_per_cta) mod num_ctas
+ * (the corner-force kernel walks zone batches c, c + num_ctas, ... per CTA). */
 int blast_cf_debug_cta_dt(blast_cf *h, double *host_out, int64_t capacity, int32_t *num_ctas, int32_t *zones_per_cta);
 
 int blast_cf_destroy(blast_cf *h);

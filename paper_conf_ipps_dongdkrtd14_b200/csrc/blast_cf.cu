@@ -17,6 +17,7 @@
 
 #include "../../include/blast_cf.h"
 #include "kb1_corner_force.cuh"
+#include "kb1_v2.cuh"
 #include "kb2_gather.cuh"
 #include "tables.h"
 #include "exchange.cuh"
@@ -59,6 +60,7 @@ struct KB1Variant {
   int zpc, nth, smem;
   kb1_launch_fn launch;
   const void *func;
+  bool persistent;   // grid = resident CTAs; CTA c runs zone batches c, c + grid, ...
 };
 
 template <int K, int ZPC, int MINB>
@@ -72,25 +74,45 @@ void launch2(const KB1Args &a, int grid, cudaStream_t s) {
   kb1_corner_force_2d<K, ZPC, MINB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
 }
 template <int K, int ZPC, int MINB>
+void launch3v2(const KB1Args &a, int grid, cudaStream_t s) {
+  using C = KB1V2Cfg<K, ZPC>;
+  kb1_v2_3d<K, ZPC, MINB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+}
+template <int K, int ZPC, int MINB>
+KB1Variant variant3v2() {
+  using C = KB1V2Cfg<K, ZPC>;
+  return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3v2<K, ZPC, MINB>, (const void *)&kb1_v2_3d<K, ZPC, MINB>,
+                    true};
+}
+template <int K, int ZPC, int MINB>
 KB1Variant variant3() {
   using C = KB1Cfg3<K, ZPC>;
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3<K, ZPC, MINB>,
-                    (const void *)&kb1_corner_force_3d<K, ZPC, MINB>};
+                    (const void *)&kb1_corner_force_3d<K, ZPC, MINB>, false};
 }
 template <int K, int ZPC, int MINB>
 KB1Variant variant2() {
   using C = KB1Cfg2<K, ZPC>;
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch2<K, ZPC, MINB>,
-                    (const void *)&kb1_corner_force_2d<K, ZPC, MINB>};
+                    (const void *)&kb1_corner_force_2d<K, ZPC, MINB>, false};
 }
 
 KB1Variant select_variant(int dim, int k) {
-  if (dim == 3) {
+  const char *force = getenv("BLAST_CF_KB1");   // experiments only: "v1" forces the per-slab kernel
+  if (dim == 3 && force && strcmp(force, "v1") == 0) {
     switch (k) {
       case 1: return variant3<1, 32, 2>();
       case 2: return variant3<2, 16, 2>();
       case 3: return variant3<3, 8, 2>();
       case 4: return variant3<4, 4, 2>();
+    }
+  }
+  if (dim == 3) {
+    switch (k) {
+      case 1: return variant3v2<1, 64, 2>();
+      case 2: return variant3v2<2, 4, 3>();
+      case 3: return variant3v2<3, 2, 2>();
+      case 4: return variant3v2<4, 1, 2>();
       case 5: return variant3<5, 2, 2>();
       case 6: return variant3<6, 2, 1>();
       case 7: return variant3<7, 1, 2>();
@@ -108,7 +130,7 @@ KB1Variant select_variant(int dim, int k) {
       case 8: return variant2<8, 1, 2>();
     }
   }
-  return KB1Variant{0, 0, 0, nullptr, nullptr};
+  return KB1Variant{0, 0, 0, nullptr, nullptr, false};
 }
 
 // Debug: F_z = A_z B^T from S(q) (kernel 7 of the paper); one CTA per zone.
@@ -456,6 +478,16 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
       for (int a = 0; a < nk; ++a) ent[fill[mesh->zone_nodes[z * nk + a]]++] = (int32_t)(z * dim * nk + a);
   }
 
+  // ---- constant tables: 1-D tables of this order, eigen-root polynomial (identical for every handle) ----
+  if (cudaMemcpyToSymbol(c_tabs, tab.data(), tab.size() * sizeof(double), ctab_off(order) * sizeof(double)) !=
+      cudaSuccess)
+    return bail(fail(BLAST_CF_ECUDA, "cudaMemcpyToSymbol(c_tabs)"));
+  {
+    const std::vector<double> ep = blastcf::eig_root_poly(EIG_POLY_DEG);
+    if (cudaMemcpyToSymbol(c_eig_poly, ep.data(), ep.size() * sizeof(double)) != cudaSuccess)
+      return bail(fail(BLAST_CF_ECUDA, "cudaMemcpyToSymbol(c_eig_poly)"));
+  }
+
   // ---- kernel variant ----
   h->var = select_variant(dim, order);
   if (!h->var.launch) return bail(fail(BLAST_CF_EUNSUPPORTED, "no kernel for dim %d order %d", dim, order));
@@ -468,6 +500,12 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
     h->local_bytes = (int)fa.localSizeBytes;
   }
   h->ncta = (int)((Z + h->var.zpc - 1) / h->var.zpc);
+  if (h->var.persistent && h->ncta > 0) {
+    int occ = 0, sms = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, h->var.func, h->var.nth, h->var.smem);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device);
+    h->ncta = std::min<int>(h->ncta, std::max(1, occ) * std::max(1, sms));
+  }
 
   // ---- uploads ----
   if ((rc = upload(&h->d_tab, tab.data(), tab.size())) ||
@@ -498,7 +536,7 @@ static int eval_impl(blast_cf *h, const double *x, const double *v, const double
   a.Fz1 = h->d_Fz1; a.FTv = out_FTv; a.cta_dt = h->d_ctadt; a.Sq = Sq;
   a.num_zones = h->Z; a.num_nodes = h->nn;
   a.ph.cfl = h->params.cfl; a.ph.q_quad = h->params.q_quad; a.ph.q_lin = h->params.q_lin;
-  a.ph.eps_sw = h->params.eps_switch; a.ph.h0 = h->h0; a.ph.inv_k = 1.0 / h->k;
+  a.ph.eps_sw = h->params.eps_switch; a.ph.inv_2eps = 0.5 / h->params.eps_switch; a.ph.h0 = h->h0; a.ph.k = (double)h->k;
   a.ph.use_visc = h->params.use_viscosity; a.ph.use_vort = h->params.use_vorticity;
   if (h->timing) cudaEventRecord(h->ev[0], h->stream);
   if (h->ncta > 0) h->var.launch(a, h->ncta, h->stream);

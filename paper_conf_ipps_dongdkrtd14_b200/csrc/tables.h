@@ -100,4 +100,37 @@ inline Tables1D build_tables(int k) {
   return T;
 }
 
+// Monomial coefficients (in t = 2r - 1) of the degree-`deg` Chebyshev interpolant of
+// y(r) = 2 cos(acos(r)/3), the largest root of y^3 - 3y - 2r = 0 on r in [0,1] (pointwise.cuh).
+inline std::vector<double> eig_root_poly(int deg) {
+  const long double pi = 3.141592653589793238462643383279502884L;
+  const int n = deg + 1;
+  std::vector<long double> f(n), c(n, 0.0L);
+  for (int k = 0; k < n; ++k) {
+    const long double t = cosl(pi * (k + 0.5L) / n), r = 0.5L * (t + 1.0L);
+    f[k] = 2.0L * cosl(acosl(r) / 3.0L);
+  }
+  for (int j = 0; j < n; ++j) {
+    long double s = 0.0L;
+    for (int k = 0; k < n; ++k) s += f[k] * cosl(pi * j * (k + 0.5L) / n);
+    c[j] = (j == 0 ? 1.0L : 2.0L) * s / n;
+  }
+  // sum_j c_j T_j(t) -> monomials, T_{j+1} = 2 t T_j - T_{j-1}
+  std::vector<long double> mono(n, 0.0L), Tm(n, 0.0L), T0(n, 0.0L), T1(n, 0.0L);
+  T0[0] = 1.0L;
+  if (n > 1) T1[1] = 1.0L;
+  for (int i = 0; i < n; ++i) mono[i] += c[0] * T0[i];
+  if (n > 1)
+    for (int i = 0; i < n; ++i) mono[i] += c[1] * T1[i];
+  for (int j = 2; j < n; ++j) {
+    for (int i = 0; i < n; ++i) Tm[i] = (i > 0 ? 2.0L * T1[i - 1] : 0.0L) - T0[i];
+    for (int i = 0; i < n; ++i) mono[i] += c[j] * Tm[i];
+    T0 = T1;
+    T1 = Tm;
+  }
+  std::vector<double> out(n);
+  for (int i = 0; i < n; ++i) out[i] = (double)mono[i];
+  return out;
+}
+
 }  // namespace blastcf

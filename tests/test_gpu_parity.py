@@ -164,9 +164,13 @@ def sampled_parity(orc, name, which, n_nodes=48, n_zones=48, seed=0):
     extra = rng.choice(m.num_zones, size=n_zones, replace=False)
     # the CTA holding the GPU's minimum dt: its zones must reproduce dt_min exactly
     cta_dt, zpc = h.debug_cta_dt()
+    ncta = len(cta_dt)
     cmin = int(np.argmin(cta_dt))
     assert cta_dt[cmin] == dt
-    arg_zones = np.arange(cmin * zpc, min((cmin + 1) * zpc, m.num_zones))
+    zone_cta = (np.arange(m.num_zones) // zpc) % ncta
+    arg_zones = np.nonzero(zone_cta == cmin)[0]
+    if len(arg_zones) > 512:   # the argmin CTA's zones: evaluate them all when cheap, else a sample + bound
+        arg_zones = arg_zones[:512]
     zones = np.unique(np.concatenate([inc, extra, arg_zones]))
     h0 = (np.prod(m.L) / m.num_zones) ** (1.0 / m.dim) / m.order   # closed form for the uniform box
     assert abs(h.info["h0"] - h0) <= 1e-14 * h0
@@ -178,9 +182,11 @@ def sampled_parity(orc, name, which, n_nodes=48, n_zones=48, seed=0):
     assert np.abs(FTv[zones] - r.FTv[pos]).max() <= TOL * np.abs(FTv).max()
     # per-CTA dt of every sampled zone's CTA must bound the oracle's zone dt, and the argmin CTA matches
     odt = r.dtz[np.searchsorted(zones, arg_zones)].min()
-    assert abs(dt - odt) <= TOL * odt, (dt, odt)
+    assert dt <= odt * (1 + TOL)
+    if (zone_cta == cmin).sum() == len(arg_zones):
+        assert abs(dt - odt) <= TOL * odt, (dt, odt)
     for z, dz in zip(zones, r.dtz):
-        assert cta_dt[z // zpc] <= dz * (1 + TOL)
+        assert cta_dt[zone_cta[z]] <= dz * (1 + TOL)
     # any-size properties
     assert np.abs(F1.sum(1)).max() <= 1e-12 * np.abs(F1).sum()
     assert abs((s.v * F1).sum() - FTv.sum()) <= 1e-12 * np.abs(s.v).max() * np.abs(F1).sum()
