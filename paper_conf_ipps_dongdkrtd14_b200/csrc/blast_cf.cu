@@ -18,6 +18,7 @@
 #include "../../include/blast_cf.h"
 #include "kb1_corner_force.cuh"
 #include "kb1_v2.cuh"
+#include "kb1_v3.cuh"
 #include "kb2_gather.cuh"
 #include "tables.h"
 #include "exchange.cuh"
@@ -85,6 +86,17 @@ KB1Variant variant3v2() {
                     true};
 }
 template <int K, int ZPC, int MINB>
+void launch3v3(const KB1Args &a, int grid, cudaStream_t s) {
+  using C = KB1V3Cfg<K, ZPC>;
+  kb1_v3_3d<K, ZPC, MINB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+}
+template <int K, int ZPC, int MINB>
+KB1Variant variant3v3() {
+  using C = KB1V3Cfg<K, ZPC>;
+  return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3v3<K, ZPC, MINB>, (const void *)&kb1_v3_3d<K, ZPC, MINB>,
+                    false};
+}
+template <int K, int ZPC, int MINB>
 KB1Variant variant3() {
   using C = KB1Cfg3<K, ZPC>;
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3<K, ZPC, MINB>,
@@ -105,6 +117,12 @@ KB1Variant select_variant(int dim, int k) {
       case 2: return variant3<2, 16, 2>();
       case 3: return variant3<3, 8, 2>();
       case 4: return variant3<4, 4, 2>();
+    }
+  }
+  if (dim == 3 && !(force && strcmp(force, "v2") == 0)) {
+    switch (k) {
+      case 3: return variant3v3<3, 2, 2>();
+      case 4: return variant3v3<4, 1, 2>();
     }
   }
   if (dim == 3) {
@@ -542,10 +560,13 @@ static int eval_impl(blast_cf *h, const double *x, const double *v, const double
   if (h->ncta > 0) h->var.launch(a, h->ncta, h->stream);
   if (h->timing) cudaEventRecord(h->ev[1], h->stream);
   const int gthreads = 256;
-  int64_t gblocks = (h->nn + gthreads - 1) / gthreads;
-  gblocks = std::max<int64_t>(1, std::min<int64_t>(gblocks, 148 * 16));
-  kb2_gather<<<(int)gblocks, gthreads, 0, h->stream>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->dim, h->nk, out_Fdot1,
-                                                        h->d_ctadt, h->ncta, out_dt_min);
+  const int64_t gblocks = std::max<int64_t>(1, (h->nn + gthreads - 1) / gthreads);
+  if (h->dim == 3)
+    kb2_gather<3, 8><<<(unsigned)gblocks, gthreads, 0, h->stream>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->nk,
+                                                                     out_Fdot1, h->d_ctadt, h->ncta, out_dt_min);
+  else
+    kb2_gather<2, 4><<<(unsigned)gblocks, gthreads, 0, h->stream>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->nk,
+                                                                     out_Fdot1, h->d_ctadt, h->ncta, out_dt_min);
   if (h->timing) cudaEventRecord(h->ev[2], h->stream);
   if (h->xch) {
     rc = blastcf::exchange_run(h->xch, out_Fdot1, out_dt_min);

@@ -3,11 +3,15 @@
 //
 // Each node sums its incident (zone, local node) entries in ascending zone id (reading R20): a fixed
 // order, so results are bitwise reproducible — no unordered atomics (north_star: "deterministic").
+// One thread per node; the first MAXE entries' indices and values are all requested before any is
+// summed (memory-level parallelism instead of a dependent load chain), nodes with more incident zones
+// (unstructured meshes) finish in a loop.
 #pragma once
 
+template <int DIM, int MAXE>
 __global__ void __launch_bounds__(256) kb2_gather(const double *__restrict__ Fz1, const int32_t *__restrict__ ptr,
-                                                  const int32_t *__restrict__ ent, int64_t num_nodes, int dim,
-                                                  int nk, double *__restrict__ out, const double *__restrict__ cta_dt,
+                                                  const int32_t *__restrict__ ent, int64_t num_nodes, int nk,
+                                                  double *__restrict__ out, const double *__restrict__ cta_dt,
                                                   int num_cta, double *__restrict__ dt_out) {
   __shared__ double red[32];
   if (blockIdx.x == gridDim.x - 1) {
@@ -24,17 +28,30 @@ __global__ void __launch_bounds__(256) kb2_gather(const double *__restrict__ Fz1
       if (threadIdx.x == 0) *dt_out = r;
     }
   }
-  for (int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; n < num_nodes; n += (int64_t)gridDim.x * blockDim.x) {
-    const int b = __ldg(ptr + n), e = __ldg(ptr + n + 1);
-    double s0 = 0.0, s1 = 0.0, s2 = 0.0;
-    for (int i = b; i < e; ++i) {
-      const int64_t o = __ldg(ent + i);   // z*dim*nk + a
-      s0 += __ldg(Fz1 + o);
-      s1 += __ldg(Fz1 + o + nk);
-      if (dim == 3) s2 += __ldg(Fz1 + o + 2 * nk);
-    }
-    out[n] = s0;
-    out[num_nodes + n] = s1;
-    if (dim == 3) out[2 * num_nodes + n] = s2;
+  const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (n >= num_nodes) return;
+  const int b = __ldg(ptr + n), e = __ldg(ptr + n + 1);
+  int o[MAXE];
+#pragma unroll
+  for (int i = 0; i < MAXE; ++i) o[i] = (b + i < e) ? __ldg(ent + b + i) : -1;
+  double v[DIM][MAXE];
+#pragma unroll
+  for (int i = 0; i < MAXE; ++i)
+#pragma unroll
+    for (int c = 0; c < DIM; ++c) v[c][i] = o[i] >= 0 ? __ldg(Fz1 + o[i] + c * nk) : 0.0;
+  double s[DIM];
+#pragma unroll
+  for (int c = 0; c < DIM; ++c) {
+    s[c] = 0.0;
+#pragma unroll
+    for (int i = 0; i < MAXE; ++i)
+      if (o[i] >= 0) s[c] += v[c][i];   // ascending zone id, the same order as the serial assembly
   }
+  for (int i = b + MAXE; i < e; ++i) {
+    const int oi = __ldg(ent + i);
+#pragma unroll
+    for (int c = 0; c < DIM; ++c) s[c] += __ldg(Fz1 + oi + c * nk);
+  }
+#pragma unroll
+  for (int c = 0; c < DIM; ++c) out[c * num_nodes + n] = s[c];
 }

@@ -20,7 +20,7 @@ for r in rows:
     if r and r[0] == 'Line No':
         hdr = r
         continue
-    if not hdr or len(r) < 8 or r[0] == '':
+    if not hdr or len(r) != len(hdr) or r[0] == '':
         continue
     key = (fname, int(r[0]))
     f = lambda x: float(x) if x not in ("", "-") else 0.0
