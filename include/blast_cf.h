@@ -84,7 +84,8 @@ void blast_cf_default_params(blast_cf_params *p);
  * blast_cf_create(mesh, order, dim)).  params NULL = defaults.  cuda_stream: a cudaStream_t (NULL =
  * the legacy default stream) on which every eval is enqueued.  nccl_unique_id: pointer to an
  * ncclUniqueId (128 bytes) shared by all ranks when mesh->nranks > 1, else NULL; the caller must have
- * selected this rank's CUDA device.  All device memory is allocated here; eval never allocates. */
+ * selected this rank's CUDA device.  All device memory is allocated here; eval never allocates.
+ * nranks > 1 with nccl_unique_id NULL creates a "loopback" handle for blast_cf_eval_loopback (tests). */
 int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_cf_params *params,
                     void *cuda_stream, const void *nccl_unique_id, blast_cf **out);
 
@@ -113,6 +114,16 @@ int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const doub
 int blast_cf_eval_debug_Fz(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
                            double *out_Fz);
 
+/* Tests only (single GPU): evaluate the n ranks of a domain decomposition on ONE device and run the
+ * shared-DOF exchange with device copies instead of NCCL — the same pack kernel, plan (ascending-rank
+ * summation) and combine kernel as the NCCL path, so partition / shared-node / ordering bugs show up
+ * on one GPU.  hs[r] must have been created with mesh->rank = r, mesh->nranks = n, nccl_unique_id
+ * NULL ("loopback" handle) and params->h0 > 0 (the global h0: no collective computes it).  Arrays are
+ * per-rank device pointers as in blast_cf_eval.  Synchronous. */
+int blast_cf_eval_loopback(blast_cf *const *hs, int n, const double *const *x, const double *const *v,
+                           const double *const *e, const double *const *rho0detJ0, double *const *out_Fdot1,
+                           double *const *out_FTv, double *const *out_dt_min);
+
 typedef struct {
   int32_t dim, order, nq, nk, nt;
   int64_t num_zones, num_nodes;
@@ -136,6 +147,10 @@ int blast_cf_kernel_times(blast_cf *h, float *ms3);
  * the stream (host_out NULL: only report the sizes).  Zone z belongs to CTA (z / zones_per_cta) mod num_ctas
  * (the corner-force kernel walks zone batches c, c + num_ctas, ... per CTA). */
 int blast_cf_debug_cta_dt(blast_cf *h, double *host_out, int64_t capacity, int32_t *num_ctas, int32_t *zones_per_cta);
+
+/* Profiling only: with BLAST_CF_PROFILE=1 in the environment at create, the corner-force kernel stamps
+ * clock64() at each of its stage barriers; copies [num_ctas][16] stamps of the last eval. */
+int blast_cf_debug_stage_clocks(blast_cf *h, long long *host_out, int64_t capacity);
 
 int blast_cf_destroy(blast_cf *h);
 const char *blast_cf_error_string(int code);

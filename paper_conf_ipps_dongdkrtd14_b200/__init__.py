@@ -93,9 +93,12 @@ def lib():
     L.blast_cf_nccl_get_unique_id.argtypes = [vp]
     L.blast_cf_exchange_plan.argtypes = [i32, i32, vp, vp, vp, i64, ctypes.POINTER(i64), vp, vp, vp]
     L.blast_cf_debug_cta_dt.argtypes = [vp, vp, i64, ctypes.POINTER(i32), ctypes.POINTER(i32)]
+    L.blast_cf_debug_stage_clocks.argtypes = [vp, vp, i64]
+    L.blast_cf_eval_loopback.argtypes = [vp, ctypes.c_int, vp, vp, vp, vp, vp, vp, vp]
     for f in ("blast_cf_create", "blast_cf_eval", "blast_cf_eval_host", "blast_cf_eval_debug_Fz", "blast_cf_get_info",
               "blast_cf_set_timing", "blast_cf_kernel_times", "blast_cf_destroy", "blast_cf_nccl_unique_id_size",
-              "blast_cf_nccl_get_unique_id", "blast_cf_exchange_plan", "blast_cf_debug_cta_dt"):
+              "blast_cf_nccl_get_unique_id", "blast_cf_exchange_plan", "blast_cf_debug_cta_dt",
+              "blast_cf_debug_stage_clocks", "blast_cf_eval_loopback"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
     return L
@@ -174,8 +177,9 @@ class CornerForce:
             m.num_neighbors = len(self._nbr[0])
             m.nbr_rank, m.nbr_offset, m.nbr_nodes = (_ptr(self._nbr[0], np.int32), _ptr(self._nbr[1], np.int64),
                                                      _ptr(self._nbr[2], np.int32))
-            assert nccl_unique_id is not None and len(nccl_unique_id) == L.blast_cf_nccl_unique_id_size()
-            uid = ctypes.create_string_buffer(bytes(nccl_unique_id), len(nccl_unique_id))
+            if nccl_unique_id is not None:   # None: loopback handle (eval_loopback, single GPU tests)
+                assert len(nccl_unique_id) == L.blast_cf_nccl_unique_id_size()
+                uid = ctypes.create_string_buffer(bytes(nccl_unique_id), len(nccl_unique_id))
         self.params = params if params is not None else default_params()
         h = ctypes.c_void_p()
         with torch.cuda.device(self.device):
@@ -259,6 +263,13 @@ class CornerForce:
                "blast_cf_debug_cta_dt")
         return out[:n.value], z.value
 
+    def debug_stage_clocks(self):
+        """[num_ctas][16] clock64 stamps at KB1's stage barriers (needs BLAST_CF_PROFILE=1 at create)."""
+        n = self.info["num_ctas"]
+        out = np.zeros((n, 16), dtype=np.int64)
+        _check(lib().blast_cf_debug_stage_clocks(self._h, out.ctypes.data, out.size), "blast_cf_debug_stage_clocks")
+        return out
+
     def set_timing(self, enable: bool):
         _check(lib().blast_cf_set_timing(self._h, int(enable)), "blast_cf_set_timing")
 
@@ -277,6 +288,19 @@ class CornerForce:
             self.close()
         except Exception:
             pass
+
+
+def eval_loopback(handles, xs, vs, es, rs):
+    """Evaluate the ranks of a loopback group on one GPU (see blast_cf_eval_loopback); returns per-rank
+    (F1, FTv, dt) tensors."""
+    n = len(handles)
+    outs = [h.alloc_outputs() for h in handles]
+    P = ctypes.c_void_p * n
+    hs = P(*[h._h for h in handles])
+    arr = lambda ts: P(*[ctypes.c_void_p(t.data_ptr()) for t in ts])
+    _check(lib().blast_cf_eval_loopback(hs, n, arr(xs), arr(vs), arr(es), arr(rs), arr([o[0] for o in outs]),
+                                        arr([o[1] for o in outs]), arr([o[2] for o in outs])), "blast_cf_eval_loopback")
+    return outs
 
 
 def nccl_unique_id() -> bytes:

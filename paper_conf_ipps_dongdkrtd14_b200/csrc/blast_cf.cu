@@ -19,6 +19,7 @@
 #include "kb1_corner_force.cuh"
 #include "kb1_v2.cuh"
 #include "kb1_v3.cuh"
+#include "kb1_v4.cuh"
 #include "kb2_gather.cuh"
 #include "tables.h"
 #include "exchange.cuh"
@@ -96,6 +97,16 @@ KB1Variant variant3v3() {
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3v3<K, ZPC, MINB>, (const void *)&kb1_v3_3d<K, ZPC, MINB>,
                     false};
 }
+template <int K>
+void launch3v4(const KB1Args &a, int grid, cudaStream_t s) {
+  using C = KB1V4Cfg<K>;
+  kb1_v4_3d<K><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+}
+template <int K>
+KB1Variant variant3v4() {
+  using C = KB1V4Cfg<K>;
+  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v4<K>, (const void *)&kb1_v4_3d<K>, true};
+}
 template <int K, int ZPC, int MINB>
 KB1Variant variant3() {
   using C = KB1Cfg3<K, ZPC>;
@@ -117,6 +128,11 @@ KB1Variant select_variant(int dim, int k) {
       case 2: return variant3<2, 16, 2>();
       case 3: return variant3<3, 8, 2>();
       case 4: return variant3<4, 4, 2>();
+    }
+  }
+  if (dim == 3 && !force) {
+    switch (k) {
+      case 4: return variant3v4<4>();
     }
   }
   if (dim == 3 && !(force && strcmp(force, "v2") == 0)) {
@@ -210,8 +226,8 @@ int nccl_get_unique_id(void *out) {
 int exchange_create(Exchange **out, const blast_cf_mesh *mesh, int dim, int64_t nn, cudaStream_t stream,
                     const void *uid) {
   *out = nullptr;
-  NcclApi *api = nccl_api();
-  if (!api) return fail(BLAST_CF_ENCCL, "cannot dlopen NCCL (set BLAST_CF_NCCL_LIB)");
+  NcclApi *api = uid ? nccl_api() : nullptr;   // uid NULL: loopback exchange (blast_cf_eval_loopback)
+  if (uid && !api) return fail(BLAST_CF_ENCCL, "cannot dlopen NCCL (set BLAST_CF_NCCL_LIB)");
   if (mesh->num_neighbors < 0 || (mesh->num_neighbors > 0 && (!mesh->nbr_rank || !mesh->nbr_offset || !mesh->nbr_nodes)))
     return fail(BLAST_CF_EINVAL, "neighbour lists");
   for (int i = 0; i < mesh->num_neighbors; ++i) {
@@ -244,6 +260,10 @@ int exchange_create(Exchange **out, const blast_cf_mesh *mesh, int dim, int64_t 
     exchange_destroy(x);
     return fail(BLAST_CF_ENOMEM, "exchange buffers");
   }
+  if (!uid) {
+    *out = x;
+    return BLAST_CF_OK;
+  }
   ncclUniqueId id;
   memcpy(&id, uid, sizeof id);
   ncclResult_t r = api->CommInitRank(&x->comm, x->nranks, id, x->rank);
@@ -267,12 +287,25 @@ int exchange_allreduce_sum2(Exchange *x, double *a, double *b) {
   return BLAST_CF_OK;
 }
 
-int exchange_run(Exchange *x, double *F1, double *dt) {
-  const int dim = x->dim;
+void exchange_pack(Exchange *x, const double *F1) {
   if (x->nrows > 0) {
     const int blocks = (int)std::min<int64_t>((x->nrows + 255) / 256, 1184);
-    xch_pack<<<blocks, 256, 0, x->stream>>>(F1, x->nn, dim, x->d_rows, x->nrows, x->d_send);
+    xch_pack<<<blocks, 256, 0, x->stream>>>(F1, x->nn, x->dim, x->d_rows, x->nrows, x->d_send);
   }
+}
+
+void exchange_combine(Exchange *x, double *F1) {
+  if (x->nu > 0) {
+    const int blocks = (int)std::min<int64_t>((x->nu + 255) / 256, 1184);
+    xch_combine<<<blocks, 256, 0, x->stream>>>(F1, x->nn, x->dim, x->d_unodes, x->nu, x->d_sptr, x->d_src, x->d_send,
+                                               x->d_recv);
+  }
+}
+
+int exchange_run(Exchange *x, double *F1, double *dt) {
+  const int dim = x->dim;
+  if (!x->comm) return BLAST_CF_OK;   // loopback: blast_cf_eval_loopback moves the data
+  exchange_pack(x, F1);
   NCCL_TRY(x->api->GroupStart(), "ncclGroupStart");
   for (int i = 0; i < x->num_nbr; ++i) {
     const int64_t o = x->nbr_offset[i], cnt = x->nbr_offset[i + 1] - o;
@@ -282,11 +315,7 @@ int exchange_run(Exchange *x, double *F1, double *dt) {
   }
   NCCL_TRY(x->api->GroupEnd(), "ncclGroupEnd");
   NCCL_TRY(x->api->AllReduce(dt, dt, 1, ncclDouble, ncclMin, x->comm, x->stream), "ncclAllReduce(min dt)");
-  if (x->nu > 0) {
-    const int blocks = (int)std::min<int64_t>((x->nu + 255) / 256, 1184);
-    xch_combine<<<blocks, 256, 0, x->stream>>>(F1, x->nn, dim, x->d_unodes, x->nu, x->d_sptr, x->d_src, x->d_send,
-                                               x->d_recv);
-  }
+  exchange_combine(x, F1);
   return BLAST_CF_OK;
 }
 
@@ -306,6 +335,7 @@ struct blast_cf {
   int32_t *d_zone_nodes = nullptr, *d_ptr = nullptr, *d_ent = nullptr;
   // host-eval staging
   double *d_in = nullptr, *d_out = nullptr;
+  long long *d_prof = nullptr;   // stage timestamps (BLAST_CF_PROFILE=1)
   // timing
   bool timing = false;
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -318,7 +348,7 @@ namespace {
 void free_handle(blast_cf *h) {
   if (!h) return;
   cudaFree(h->d_tab); cudaFree(h->d_J0inv); cudaFree(h->d_gamma); cudaFree(h->d_Fz1); cudaFree(h->d_ctadt);
-  cudaFree(h->d_zone_nodes); cudaFree(h->d_ptr); cudaFree(h->d_ent); cudaFree(h->d_in); cudaFree(h->d_out);
+  cudaFree(h->d_zone_nodes); cudaFree(h->d_ptr); cudaFree(h->d_ent); cudaFree(h->d_in); cudaFree(h->d_out); cudaFree(h->d_prof);
   for (auto &e : h->ev)
     if (e) cudaEventDestroy(e);
   if (h->xch) blastcf::exchange_destroy(h->xch);
@@ -388,7 +418,8 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
   if (mesh->num_zones > 0 && (!mesh->zone_nodes || !mesh->x0)) return fail(BLAST_CF_EINVAL, "zone_nodes/x0 NULL");
   if (!mesh->mat_gamma || mesh->num_mats < 1) return fail(BLAST_CF_EINVAL, "mat_gamma/num_mats");
   const int nranks = mesh->nranks < 1 ? 1 : mesh->nranks;
-  if (nranks > 1 && !nccl_unique_id) return fail(BLAST_CF_EINVAL, "nranks > 1 needs nccl_unique_id");
+  if (nranks > 1 && !nccl_unique_id && !(params && params->h0 > 0.0))
+    return fail(BLAST_CF_EINVAL, "nranks > 1 without nccl_unique_id (loopback) needs params->h0 > 0");
 
   blast_cf *h = new (std::nothrow) blast_cf();
   if (!h) return fail(BLAST_CF_ENOMEM, "host allocation");
@@ -480,8 +511,10 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
   if (nranks > 1) {
     rc = blastcf::exchange_create(&h->xch, mesh, dim, nn, h->stream, nccl_unique_id);
     if (rc) { free_handle(h); return rc; }
-    rc = blastcf::exchange_allreduce_sum2(h->xch, &gvol, &gz);
-    if (rc) { free_handle(h); return rc; }
+    if (nccl_unique_id) {
+      rc = blastcf::exchange_allreduce_sum2(h->xch, &gvol, &gz);
+      if (rc) { free_handle(h); return rc; }
+    }
   }
   h->h0 = h->params.h0 > 0.0 ? h->params.h0 : pow(gvol / gz, 1.0 / dim) / order;
 
@@ -537,6 +570,8 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
     return bail(fail(BLAST_CF_ENOMEM, "workspace allocation"));
   for (auto &e : h->ev)
     if (cudaEventCreate(&e) != cudaSuccess) return bail(fail(BLAST_CF_ECUDA, "event create"));
+  if (getenv("BLAST_CF_PROFILE") && cudaMalloc(&h->d_prof, std::max(h->ncta, 1) * 16 * sizeof(long long)) != cudaSuccess)
+    return bail(fail(BLAST_CF_ENOMEM, "profile buffer"));
   *out = h;
   return BLAST_CF_OK;
 }
@@ -551,7 +586,7 @@ static int eval_impl(blast_cf *h, const double *x, const double *v, const double
   KB1Args a;
   a.x = x; a.v = v; a.e = e; a.rho0detJ0 = rho0detJ0;
   a.zone_nodes = h->d_zone_nodes; a.J0inv = h->d_J0inv; a.zone_gamma = h->d_gamma; a.tab = h->d_tab;
-  a.Fz1 = h->d_Fz1; a.FTv = out_FTv; a.cta_dt = h->d_ctadt; a.Sq = Sq;
+  a.Fz1 = h->d_Fz1; a.FTv = out_FTv; a.cta_dt = h->d_ctadt; a.Sq = Sq; a.prof = h->d_prof;
   a.num_zones = h->Z; a.num_nodes = h->nn;
   a.ph.cfl = h->params.cfl; a.ph.q_quad = h->params.q_quad; a.ph.q_lin = h->params.q_lin;
   a.ph.eps_sw = h->params.eps_switch; a.ph.inv_2eps = 0.5 / h->params.eps_switch; a.ph.h0 = h->h0; a.ph.k = (double)h->k;
@@ -622,6 +657,54 @@ int blast_cf_eval_debug_Fz(blast_cf *h, const double *x, const double *v, const 
   return rc;
 }
 
+int blast_cf_eval_loopback(blast_cf *const *hs, int n, const double *const *x, const double *const *v,
+                           const double *const *e, const double *const *rho0detJ0, double *const *out_Fdot1,
+                           double *const *out_FTv, double *const *out_dt_min) {
+  if (!hs || n < 1 || !x || !v || !e || !rho0detJ0 || !out_Fdot1 || !out_FTv || !out_dt_min)
+    return fail(BLAST_CF_EINVAL, "NULL argument");
+  for (int r = 0; r < n; ++r) {
+    if (!hs[r] || !hs[r]->xch || hs[r]->xch->comm || hs[r]->xch->nranks != n || hs[r]->xch->rank != r)
+      return fail(BLAST_CF_EINVAL, "handle %d is not rank %d of a %d-rank loopback group", r, r, n);
+  }
+  int rc;
+  // 1. local corner force + gather on every partition, 2. pack shared-node partials
+  for (int r = 0; r < n; ++r) {
+    if ((rc = eval_impl(hs[r], x[r], v[r], e[r], rho0detJ0[r], out_Fdot1[r], out_FTv[r], out_dt_min[r], nullptr)))
+      return rc;
+    blastcf::exchange_pack(hs[r]->xch, out_Fdot1[r]);
+  }
+  for (int r = 0; r < n; ++r) CUDA_TRY(cudaStreamSynchronize(hs[r]->stream));
+  // 3. the exchange: rank r's recv rows from q are rank q's send rows for r (same order: global node id)
+  for (int r = 0; r < n; ++r) {
+    blastcf::Exchange *xr = hs[r]->xch;
+    for (int i = 0; i < xr->num_nbr; ++i) {
+      const int q = xr->nbr_rank[i];
+      blastcf::Exchange *xq = hs[q]->xch;
+      int iq = -1;
+      for (int t = 0; t < xq->num_nbr; ++t)
+        if (xq->nbr_rank[t] == r) iq = t;
+      const int64_t cnt = xr->nbr_offset[i + 1] - xr->nbr_offset[i];
+      if (iq < 0 || xq->nbr_offset[iq + 1] - xq->nbr_offset[iq] != cnt)
+        return fail(BLAST_CF_EINVAL, "ranks %d and %d disagree on their shared nodes", r, q);
+      CUDA_TRY(cudaMemcpy(xr->d_recv + xr->nbr_offset[i] * xr->dim, xq->d_send + xq->nbr_offset[iq] * xq->dim,
+                          cnt * xr->dim * sizeof(double), cudaMemcpyDeviceToDevice));
+    }
+  }
+  // 4. global min dt
+  double dtg = HUGE_VAL, d;
+  for (int r = 0; r < n; ++r) {
+    CUDA_TRY(cudaMemcpy(&d, out_dt_min[r], sizeof d, cudaMemcpyDeviceToHost));
+    dtg = std::min(dtg, d);
+  }
+  // 5. ordered combine on every rank
+  for (int r = 0; r < n; ++r) {
+    CUDA_TRY(cudaMemcpy(out_dt_min[r], &dtg, sizeof dtg, cudaMemcpyHostToDevice));
+    blastcf::exchange_combine(hs[r]->xch, out_Fdot1[r]);
+    CUDA_TRY(cudaStreamSynchronize(hs[r]->stream));
+  }
+  return check_async(hs[0]);
+}
+
 int blast_cf_get_info(const blast_cf *h, blast_cf_info *info) {
   if (!h || !info) return fail(BLAST_CF_EINVAL, "NULL argument");
   info->dim = h->dim; info->order = h->k; info->nq = h->nq; info->nk = h->nk; info->nt = h->nt;
@@ -660,6 +743,15 @@ int blast_cf_debug_cta_dt(blast_cf *h, double *host_out, int64_t capacity, int32
     CUDA_TRY(cudaStreamSynchronize(h->stream));
     CUDA_TRY(cudaMemcpy(host_out, h->d_ctadt, h->ncta * sizeof(double), cudaMemcpyDeviceToHost));
   }
+  return BLAST_CF_OK;
+}
+
+int blast_cf_debug_stage_clocks(blast_cf *h, long long *host_out, int64_t capacity) {
+  if (!h || !host_out) return fail(BLAST_CF_EINVAL, "NULL argument");
+  if (!h->d_prof) return fail(BLAST_CF_EINVAL, "set BLAST_CF_PROFILE=1 before create");
+  if (capacity < (int64_t)h->ncta * 16) return fail(BLAST_CF_EINVAL, "capacity");
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  CUDA_TRY(cudaMemcpy(host_out, h->d_prof, (size_t)h->ncta * 16 * sizeof(long long), cudaMemcpyDeviceToHost));
   return BLAST_CF_OK;
 }
 

@@ -159,12 +159,14 @@ inline void exchange_destroy(Exchange *x) {
   delete x;
 }
 
-inline int exchange_kernels(const Exchange *x) { return x->nrows > 0 ? 2 : 0; }
+inline int exchange_kernels(const Exchange *x) { return (x->nrows > 0 ? 1 : 0) + (x->nu > 0 ? 1 : 0); }
 
 int exchange_create(Exchange **out, const blast_cf_mesh *mesh, int dim, int64_t nn, cudaStream_t stream,
                     const void *uid);
 int exchange_allreduce_sum2(Exchange *x, double *a, double *b);
 int exchange_run(Exchange *x, double *F1, double *dt);
+void exchange_pack(Exchange *x, const double *F1);
+void exchange_combine(Exchange *x, double *F1);
 int nccl_get_unique_id(void *out);
 
 }  // namespace blastcf

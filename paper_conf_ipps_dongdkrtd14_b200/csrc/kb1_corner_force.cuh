@@ -25,6 +25,7 @@ struct KB1Args {
   double *FTv;             // [Z][NT]
   double *cta_dt;          // [gridDim.x]
   double *Sq;              // debug only (tests): S(q) = alpha sigma adj(J)^T as [Z][NQ][D*D], else nullptr
+  long long *prof;         // debug only: per-CTA clock64 stamps at the stage barriers [grid][16], else nullptr
   int64_t num_zones, num_nodes;
   CFPhys ph;
 };

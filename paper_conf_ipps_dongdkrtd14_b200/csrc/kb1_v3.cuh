@@ -70,6 +70,13 @@ __global__ void __launch_bounds__(KB1V3Cfg<K, ZPC>::NTH, MINB) kb1_v3_3d(const K
   double *sRed = sZone + ZPC * Dm::ZONE;
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  int nstamp = 0;
+#define KB1_STAMP()                                                                       \
+  do {                                                                                    \
+    if (a.prof != nullptr && tid == 0) a.prof[blockIdx.x * 16 + nstamp] = clock64();      \
+    ++nstamp;                                                                             \
+  } while (0)
+  KB1_STAMP();
   const int lr = lane >> 2, lc = lane & 3;              // fragment row / k-column of this lane
   const int64_t zone0 = (int64_t)blockIdx.x * ZPC;
   const int64_t Z = a.num_zones, nn = a.num_nodes;
@@ -106,6 +113,7 @@ __global__ void __launch_bounds__(KB1V3Cfg<K, ZPC>::NTH, MINB) kb1_v3_3d(const K
     sZone[zl * Dm::ZONE + Dm::R0 + Dm::R1 + r] = val;
   }
   __syncthreads();
+  KB1_STAMP();
 
   // Index clamping instead of bounds tests: a padded k (or column) reads a valid neighbour whose A-fragment
   // coefficient is zero (or whose output is discarded), so every B-fragment load is unconditional.
@@ -161,6 +169,7 @@ __global__ void __launch_bounds__(KB1V3Cfg<K, ZPC>::NTH, MINB) kb1_v3_3d(const K
     }
   }
   __syncthreads();
+  KB1_STAMP();
 
   // ---- stage B: U0 = B.TB, U1 = G.TB, U2 = B.TG over a1 -> q1 (columns (f, q2, a0)); UE = Phi.TE --------
   {
@@ -213,6 +222,7 @@ __global__ void __launch_bounds__(KB1V3Cfg<K, ZPC>::NTH, MINB) kb1_v3_3d(const K
     }
   }
   __syncthreads();
+  KB1_STAMP();
 
   // ---- stage C (a0 -> q0, DFMA) + point evaluation, two points per thread --------------------------
   const int my_zl = tid / TPZ, pr = tid - my_zl * TPZ;
@@ -276,13 +286,15 @@ __global__ void __launch_bounds__(KB1V3Cfg<K, ZPC>::NTH, MINB) kb1_v3_3d(const K
       }
     }
   }
-  __syncthreads();   // every U read is done
+  __syncthreads();
+  KB1_STAMP();   // every U read is done
   if (has_point) {
     double *SBp = sZone + my_zl * Dm::ZONE + Dm::R0 + Dm::O_SB + (q2 * N + q1) * NH + q0a;
 #pragma unroll
     for (int cd = 0; cd < 10; ++cd) SBp[cd * N2 * NH] = SB[cd];
   }
   __syncthreads();
+  KB1_STAMP();
 
   // transposed table fragments for the back stages (reloaded here: not kept live through the point stage)
   double fBt[KS_N], fGt[KS_N], fPt[KS_N];
@@ -322,6 +334,7 @@ __global__ void __launch_bounds__(KB1V3Cfg<K, ZPC>::NTH, MINB) kb1_v3_3d(const K
     }
   }
   __syncthreads();
+  KB1_STAMP();
 
   // ---- stage B^T: ZB[c][q2][a1][a0] = sum_q1 B[q1][a1] Y_c0 + G[q1][a1] Y_c1 ; ZG = sum_q1 B[q1][a1] Y_c2
   //      (columns (q2, a0)); ZE[q2][j1][j0] = sum_q1 Phi[q1][j1] YE[j0][q2][q1] (columns (q2, j0)) --------
@@ -372,6 +385,7 @@ __global__ void __launch_bounds__(KB1V3Cfg<K, ZPC>::NTH, MINB) kb1_v3_3d(const K
     }
   }
   __syncthreads();
+  KB1_STAMP();
 
   // ---- stage A^T: F_c[a2][aa] = sum_q2 B[q2][a2] ZB_c[q2][aa] + G[q2][a2] ZG_c[q2][aa] -> global;
   //      FTv[j2][jj] = sum_q2 Phi[q2][j2] ZE[q2][jj] -> global ------------------------------------------
@@ -418,4 +432,6 @@ __global__ void __launch_bounds__(KB1V3Cfg<K, ZPC>::NTH, MINB) kb1_v3_3d(const K
   if (bad) dtmin = 0.0;
   const double m = block_min(dtmin, sRed);
   if (tid == 0) a.cta_dt[blockIdx.x] = m;
+  KB1_STAMP();
+#undef KB1_STAMP
 }
