@@ -50,6 +50,14 @@ struct KB1V4Cfg {
   static constexpr int SMEM_BYTES = Dm::TOTAL * 8;
 };
 
+// thread index read through asm volatile: stops the compiler from hoisting every stage's index arithmetic
+// out of the persistent zone loop (which pins registers and spills in the 88-register DMMA warps)
+__device__ __forceinline__ int opaque_tid() {
+  int t;
+  asm volatile("mov.u32 %0, %%tid.x;" : "=r"(t));
+  return t;
+}
+
 __device__ __forceinline__ void kw_bar() { asm volatile("bar.sync 1, 256;\n" ::: "memory"); }
 
 template <int K>
@@ -104,6 +112,7 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
   };
   // forward stages A and B of the zone in XE -> U buffer ub (+ J0/gamma -> sJ slot js)
   auto kw_forward = [&](double *ub, double *js) {
+    const int ktid = opaque_tid() - NPW, kwarp = ktid >> 5, lr = (ktid & 31) >> 2, lc = ktid & 3;
     double fB[KS_P], fG[KS_P], fP[KS_T];
 #pragma unroll
     for (int s = 0; s < KS_P; ++s) {
@@ -114,86 +123,108 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
     for (int s = 0; s < KS_T; ++s) fP[s] = tfrag<false>(tPhi, T, N, T, lr, 4 * s + lc);
     if (ktid < 10) js[ktid] = sXE[Dm::XE_J + ktid];
     double *Tr = sWk;
-    {   // stage A
-      constexpr int NC = 6 * P2, NTL = (NC + 7) / 8, NCE = T2, NTE = (NCE + 7) / 8;
-      for (int j = kwarp; j < NTL + NTE; j += NKWW) {
-        if (j < NTL) {
-          const int nb = min(j * 8 + lr, NC - 1);
-          const int fb = nb / P2, ab_ = nb - fb * P2;
-          const double *Xb = sXE + Dm::XE_X + fb * P3 + ab_;
-          double db0 = 0.0, db1 = 0.0, dg0 = 0.0, dg1 = 0.0;
+    {   // stage A: each warp takes tiles kwarp, kwarp + 8, ... of the 6 P^2 columns at once (loads first)
+      constexpr int NC = 6 * P2, NTL = (NC + 7) / 8, JPW = (NTL + NKWW - 1) / NKWW;
+      double bx[JPW][KS_P];
 #pragma unroll
-          for (int s = 0; s < KS_P; ++s) {
-            const double b = Xb[min(4 * s + lc, P - 1) * P2];
-            dmma(db0, db1, fB[s], b);
-            dmma(dg0, dg1, fG[s], b);
+      for (int t = 0; t < JPW; ++t) {
+        const int nb = min((kwarp + t * NKWW) * 8 + lr, NC - 1);
+        const int fb = nb / P2, ab_ = nb - fb * P2;
+#pragma unroll
+        for (int s = 0; s < KS_P; ++s) bx[t][s] = sXE[Dm::XE_X + fb * P3 + min(4 * s + lc, P - 1) * P2 + ab_];
+      }
+      double db[JPW][2], dg[JPW][2];
+#pragma unroll
+      for (int t = 0; t < JPW; ++t) {
+        db[t][0] = db[t][1] = dg[t][0] = dg[t][1] = 0.0;
+#pragma unroll
+        for (int s = 0; s < KS_P; ++s) {
+          dmma(db[t][0], db[t][1], fB[s], bx[t][s]);
+          dmma(dg[t][0], dg[t][1], fG[s], bx[t][s]);
+        }
+      }
+#pragma unroll
+      for (int t = 0; t < JPW; ++t) {
+        const int j = kwarp + t * NKWW;
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+          const int n = j * 8 + 2 * lc + i;
+          if (j < NTL && lr < N && n < NC) {
+            const int f = n / P2, aa = n - f * P2;
+            Tr[Dm::O_T + (f * 2 + 0) * N * P2 + lr * P2 + aa] = db[t][i];
+            Tr[Dm::O_T + (f * 2 + 1) * N * P2 + lr * P2 + aa] = dg[t][i];
           }
+        }
+      }
+      constexpr int NCE = T2, NTE = (NCE + 7) / 8;   // TE = Phi . E (few tiles)
+      for (int te = kwarp; te < NTE; te += NKWW) {
+        const int nb = min(te * 8 + lr, NCE - 1);
+        double d0 = 0.0, d1 = 0.0;
 #pragma unroll
-          for (int i = 0; i < 2; ++i) {
-            const int n = j * 8 + 2 * lc + i;
-            if (lr < N && n < NC) {
-              const int f = n / P2, aa = n - f * P2;
-              Tr[Dm::O_T + (f * 2 + 0) * N * P2 + lr * P2 + aa] = i ? db1 : db0;
-              Tr[Dm::O_T + (f * 2 + 1) * N * P2 + lr * P2 + aa] = i ? dg1 : dg0;
-            }
-          }
-        } else {
-          const int te = j - NTL;
-          const int nb = min(te * 8 + lr, NCE - 1);
-          double d0 = 0.0, d1 = 0.0;
+        for (int s = 0; s < KS_T; ++s) dmma(d0, d1, fP[s], sXE[Dm::XE_E + min(4 * s + lc, T - 1) * T2 + nb]);
 #pragma unroll
-          for (int s = 0; s < KS_T; ++s) dmma(d0, d1, fP[s], sXE[Dm::XE_E + min(4 * s + lc, T - 1) * T2 + nb]);
-#pragma unroll
-          for (int i = 0; i < 2; ++i) {
-            const int n = te * 8 + 2 * lc + i;
-            if (lr < N && n < NCE) Tr[Dm::O_TE + lr * T2 + n] = i ? d1 : d0;
-          }
+        for (int i = 0; i < 2; ++i) {
+          const int n = te * 8 + 2 * lc + i;
+          if (lr < N && n < NCE) Tr[Dm::O_TE + lr * T2 + n] = i ? d1 : d0;
         }
       }
     }
     kw_bar();
-    {   // stage B
-      constexpr int NC = 6 * N * P, NTL = (NC + 7) / 8, NCE = N * T, NTE = (NCE + 7) / 8;
-      for (int j = kwarp; j < NTL + NTE; j += NKWW) {
-        if (j < NTL) {
-          const int nb = min(j * 8 + lr, NC - 1);
-          const int fb = nb / (N * P), rb = nb - fb * (N * P), q2b = rb / P, a0b = rb - q2b * P;
-          const double *TBb = Tr + Dm::O_T + ((fb * 2 + 0) * N + q2b) * P2 + a0b;
-          const double *TGb = TBb + N * P2;
-          double u00 = 0.0, u01 = 0.0, u10 = 0.0, u11 = 0.0, u20 = 0.0, u21 = 0.0;
+    {   // stage B: U0 = B.TB, U1 = G.TB, U2 = B.TG; tiles kwarp, kwarp + 8, ... at once
+      constexpr int NC = 6 * N * P, NTL = (NC + 7) / 8, JPW = (NTL + NKWW - 1) / NKWW;
+      double tb[JPW][KS_P], tg[JPW][KS_P];
 #pragma unroll
-          for (int s = 0; s < KS_P; ++s) {
-            const int a1 = min(4 * s + lc, P - 1);
-            const double tb = TBb[a1 * P], tg = TGb[a1 * P];
-            dmma(u00, u01, fB[s], tb);
-            dmma(u10, u11, fG[s], tb);
-            dmma(u20, u21, fB[s], tg);
+      for (int t = 0; t < JPW; ++t) {
+        const int nb = min((kwarp + t * NKWW) * 8 + lr, NC - 1);
+        const int fb = nb / (N * P), rb = nb - fb * (N * P), q2b = rb / P, a0b = rb - q2b * P;
+        const double *TBb = Tr + Dm::O_T + ((fb * 2 + 0) * N + q2b) * P2 + a0b;
+#pragma unroll
+        for (int s = 0; s < KS_P; ++s) {
+          const int a1 = min(4 * s + lc, P - 1);
+          tb[t][s] = TBb[a1 * P];
+          tg[t][s] = TBb[N * P2 + a1 * P];
+        }
+      }
+      double u[JPW][3][2];
+#pragma unroll
+      for (int t = 0; t < JPW; ++t) {
+#pragma unroll
+        for (int m = 0; m < 3; ++m) u[t][m][0] = u[t][m][1] = 0.0;
+#pragma unroll
+        for (int s = 0; s < KS_P; ++s) {
+          dmma(u[t][0][0], u[t][0][1], fB[s], tb[t][s]);
+          dmma(u[t][1][0], u[t][1][1], fG[s], tb[t][s]);
+          dmma(u[t][2][0], u[t][2][1], fB[s], tg[t][s]);
+        }
+      }
+#pragma unroll
+      for (int t = 0; t < JPW; ++t) {
+        const int j = kwarp + t * NKWW;
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+          const int n = j * 8 + 2 * lc + i;
+          if (j < NTL && lr < N && n < NC) {
+            const int f = n / (N * P), rr = n - f * (N * P), q2 = rr / P, a0 = rr - q2 * P;
+            double *U = ub + (((f * 3) * N + q2) * N + lr) * P + a0;
+            U[0] = u[t][0][i];
+            U[N2 * P] = u[t][1][i];
+            U[2 * N2 * P] = u[t][2][i];
           }
+        }
+      }
+      constexpr int NCE = N * T, NTE = (NCE + 7) / 8;   // UE = Phi . TE
+      for (int te = kwarp; te < NTE; te += NKWW) {
+        const int nb = min(te * 8 + lr, NCE - 1);
+        const int q2b = nb / T, j0b = nb - q2b * T;
+        double d0 = 0.0, d1 = 0.0;
 #pragma unroll
-          for (int i = 0; i < 2; ++i) {
-            const int n = j * 8 + 2 * lc + i;
-            if (lr < N && n < NC) {
-              const int f = n / (N * P), rr = n - f * (N * P), q2 = rr / P, a0 = rr - q2 * P;
-              double *U = ub + (((f * 3) * N + q2) * N + lr) * P + a0;
-              U[0] = i ? u01 : u00;
-              U[N2 * P] = i ? u11 : u10;
-              U[2 * N2 * P] = i ? u21 : u20;
-            }
-          }
-        } else {
-          const int te = j - NTL;
-          const int nb = min(te * 8 + lr, NCE - 1);
-          const int q2b = nb / T, j0b = nb - q2b * T;
-          double d0 = 0.0, d1 = 0.0;
+        for (int s = 0; s < KS_T; ++s) dmma(d0, d1, fP[s], Tr[Dm::O_TE + q2b * T2 + min(4 * s + lc, T - 1) * T + j0b]);
 #pragma unroll
-          for (int s = 0; s < KS_T; ++s) dmma(d0, d1, fP[s], Tr[Dm::O_TE + q2b * T2 + min(4 * s + lc, T - 1) * T + j0b]);
-#pragma unroll
-          for (int i = 0; i < 2; ++i) {
-            const int n = te * 8 + 2 * lc + i;
-            if (lr < N && n < NCE) {
-              const int q2 = n / T, j0 = n - q2 * T;
-              ub[Dm::O_UE + (q2 * N + lr) * T + j0] = i ? d1 : d0;
-            }
+        for (int i = 0; i < 2; ++i) {
+          const int n = te * 8 + 2 * lc + i;
+          if (lr < N && n < NCE) {
+            const int q2 = n / T, j0 = n - q2 * T;
+            ub[Dm::O_UE + (q2 * N + lr) * T + j0] = i ? d1 : d0;
           }
         }
       }
@@ -201,6 +232,7 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
   };
   // back stages C^T, B^T, A^T of zone z from the S buffer sb
   auto kw_back = [&](const double *sb, int64_t z) {
+    const int ktid = opaque_tid() - NPW, kwarp = ktid >> 5, lr = (ktid & 31) >> 2, lc = ktid & 3;
     double fBt[KS_N], fGt[KS_N], fPt[KS_N];
 #pragma unroll
     for (int s = 0; s < KS_N; ++s) {
@@ -209,104 +241,152 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
       fPt[s] = tfrag<true>(tPhi, T, N, T, lr, 4 * s + lc);
     }
     double *Wr = sWk;
-    {   // C^T: Y[cd][a0][col] and YE[j0][col], col = q2*N + q1
+    {   // C^T: each warp takes one column tile (col = q2*N + q1), five matrices at a time
       constexpr int NTL = (N2 + 7) / 8;
-      for (int j = kwarp; j < 10 * NTL; j += NKWW) {
-        const int cd = j / NTL, tl = j - cd * NTL;
+      for (int tl = kwarp; tl < NTL; tl += NKWW) {
         const int colb = min(tl * 8 + lr, N2 - 1);
-        const double *Sc = sb + cd * N3 + colb * N;
-        double d0 = 0.0, d1 = 0.0;
 #pragma unroll
-        for (int s = 0; s < KS_N; ++s)
-          dmma(d0, d1, cd == 9 ? fPt[s] : (cd % 3 == 0 ? fGt[s] : fBt[s]), Sc[min(4 * s + lc, N - 1)]);
+        for (int h = 0; h < 2; ++h) {
+          double sv[5][KS_N];
 #pragma unroll
-        for (int i = 0; i < 2; ++i) {
-          const int col = tl * 8 + 2 * lc + i;
-          if (col < N2) {
-            if (cd < 9 && lr < P) Wr[Dm::O_Y + (cd * P + lr) * N2 + col] = i ? d1 : d0;
-            if (cd == 9 && lr < T) Wr[Dm::O_YE + lr * N2 + col] = i ? d1 : d0;
+          for (int c5 = 0; c5 < 5; ++c5)
+#pragma unroll
+            for (int s = 0; s < KS_N; ++s) sv[c5][s] = sb[(h * 5 + c5) * N3 + colb * N + min(4 * s + lc, N - 1)];
+          double d[5][2];
+#pragma unroll
+          for (int c5 = 0; c5 < 5; ++c5) {
+            const int cd = h * 5 + c5;
+            d[c5][0] = d[c5][1] = 0.0;
+#pragma unroll
+            for (int s = 0; s < KS_N; ++s)
+              dmma(d[c5][0], d[c5][1], cd == 9 ? fPt[s] : (cd % 3 == 0 ? fGt[s] : fBt[s]), sv[c5][s]);
+          }
+#pragma unroll
+          for (int i = 0; i < 2; ++i) {
+            const int col = tl * 8 + 2 * lc + i;
+            if (col < N2) {
+#pragma unroll
+              for (int c5 = 0; c5 < 5; ++c5) {
+                const int cd = h * 5 + c5;
+                if (cd < 9 && lr < P) Wr[Dm::O_Y + (cd * P + lr) * N2 + col] = d[c5][i];
+                if (cd == 9 && lr < T) Wr[Dm::O_YE + lr * N2 + col] = d[c5][i];
+              }
+            }
           }
         }
       }
     }
     kw_bar();
-    {   // B^T
-      constexpr int NC = N * P, NTL = (NC + 7) / 8, NCE = N * T, NTE = (NCE + 7) / 8;
-      for (int j = kwarp; j < 3 * NTL + NTE; j += NKWW) {
-        if (j < 3 * NTL) {
-          const int c = j / NTL, tl = j - c * NTL;
-          const int nb = min(tl * 8 + lr, NC - 1);
-          const int q2b = nb / P, a0b = nb - q2b * P;
-          const double *Yb = Wr + Dm::O_Y + (c * 3 * P + a0b) * N2 + q2b * N;
-          double zb0 = 0.0, zb1 = 0.0, zg0 = 0.0, zg1 = 0.0;
+    {   // B^T: jobs (c, tile) spread over the warps, each warp's jobs loaded/multiplied/stored together
+      constexpr int NC = N * P, NTL = (NC + 7) / 8, NJ = 3 * NTL, JPW = (NJ + NKWW - 1) / NKWW;
+      double y[JPW][3][KS_N];
 #pragma unroll
-          for (int s = 0; s < KS_N; ++s) {
-            const int q1 = min(4 * s + lc, N - 1);
-            dmma(zb0, zb1, fBt[s], Yb[q1]);
-            dmma(zb0, zb1, fGt[s], Yb[P * N2 + q1]);
-            dmma(zg0, zg1, fBt[s], Yb[2 * P * N2 + q1]);
+      for (int t = 0; t < JPW; ++t) {
+        const int j = min(kwarp + t * NKWW, NJ - 1);
+        const int c = j / NTL, tl = j - c * NTL;
+        const int nb = min(tl * 8 + lr, NC - 1);
+        const int q2b = nb / P, a0b = nb - q2b * P;
+        const double *Yb = Wr + Dm::O_Y + (c * 3 * P + a0b) * N2 + q2b * N;
+#pragma unroll
+        for (int s = 0; s < KS_N; ++s) {
+          const int q1 = min(4 * s + lc, N - 1);
+          y[t][0][s] = Yb[q1];
+          y[t][1][s] = Yb[P * N2 + q1];
+          y[t][2][s] = Yb[2 * P * N2 + q1];
+        }
+      }
+      double zb[JPW][2], zg[JPW][2];
+#pragma unroll
+      for (int t = 0; t < JPW; ++t) {
+        zb[t][0] = zb[t][1] = zg[t][0] = zg[t][1] = 0.0;
+#pragma unroll
+        for (int s = 0; s < KS_N; ++s) {
+          dmma(zb[t][0], zb[t][1], fBt[s], y[t][0][s]);
+          dmma(zb[t][0], zb[t][1], fGt[s], y[t][1][s]);
+          dmma(zg[t][0], zg[t][1], fBt[s], y[t][2][s]);
+        }
+      }
+#pragma unroll
+      for (int t = 0; t < JPW; ++t) {
+        const int j = kwarp + t * NKWW;
+        const int c = j / NTL, tl = j - c * NTL;
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+          const int n = tl * 8 + 2 * lc + i;
+          if (j < NJ && lr < P && n < NC) {
+            const int q2 = n / P, a0 = n - q2 * P;
+            Wr[Dm::O_Z + ((c * 2 + 0) * N + q2) * P2 + lr * P + a0] = zb[t][i];
+            Wr[Dm::O_Z + ((c * 2 + 1) * N + q2) * P2 + lr * P + a0] = zg[t][i];
           }
+        }
+      }
+      constexpr int NCE = N * T, NTE = (NCE + 7) / 8;   // ZE = Phi^T . YE
+      for (int te = kwarp; te < NTE; te += NKWW) {
+        const int nb = min(te * 8 + lr, NCE - 1);
+        const int q2b = nb / T, j0b = nb - q2b * T;
+        double d0 = 0.0, d1 = 0.0;
+#pragma unroll
+        for (int s = 0; s < KS_N; ++s) dmma(d0, d1, fPt[s], Wr[Dm::O_YE + j0b * N2 + q2b * N + min(4 * s + lc, N - 1)]);
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+          const int n = te * 8 + 2 * lc + i;
+          if (lr < T && n < NCE) {
+            const int q2 = n / T, j0 = n - q2 * T;
+            Wr[Dm::O_ZE + q2 * T2 + lr * T + j0] = i ? d1 : d0;
+          }
+        }
+      }
+    }
+    kw_bar();
+    {   // A^T -> global: jobs (c, tile) and the F^T v tiles, each warp's jobs loaded/multiplied/stored together
+      constexpr int NTL = (P2 + 7) / 8, NJ = 3 * NTL, JPW = (NJ + NKWW - 1) / NKWW;
+      double zv[JPW][2][KS_N];
+#pragma unroll
+      for (int t = 0; t < JPW; ++t) {
+        const int j = min(kwarp + t * NKWW, NJ - 1);
+        const int c = j / NTL, tl = j - c * NTL;
+        const int nb = min(tl * 8 + lr, P2 - 1);
+        const double *Zb = Wr + Dm::O_Z + c * 2 * N * P2 + nb;
+#pragma unroll
+        for (int s = 0; s < KS_N; ++s) {
+          const int q2 = min(4 * s + lc, N - 1);
+          zv[t][0][s] = Zb[q2 * P2];
+          zv[t][1][s] = Zb[(N + q2) * P2];
+        }
+      }
+      double d[JPW][2];
+#pragma unroll
+      for (int t = 0; t < JPW; ++t) {
+        d[t][0] = d[t][1] = 0.0;
+#pragma unroll
+        for (int s = 0; s < KS_N; ++s) {
+          dmma(d[t][0], d[t][1], fBt[s], zv[t][0][s]);
+          dmma(d[t][0], d[t][1], fGt[s], zv[t][1][s]);
+        }
+      }
+#pragma unroll
+      for (int t = 0; t < JPW; ++t) {
+        const int j = kwarp + t * NKWW;
+        const int c = j / NTL, tl = j - c * NTL;
+        if (j < NJ && lr < P) {
 #pragma unroll
           for (int i = 0; i < 2; ++i) {
             const int n = tl * 8 + 2 * lc + i;
-            if (lr < P && n < NC) {
-              const int q2 = n / P, a0 = n - q2 * P;
-              Wr[Dm::O_Z + ((c * 2 + 0) * N + q2) * P2 + lr * P + a0] = i ? zb1 : zb0;
-              Wr[Dm::O_Z + ((c * 2 + 1) * N + q2) * P2 + lr * P + a0] = i ? zg1 : zg0;
-            }
-          }
-        } else {
-          const int te = j - 3 * NTL;
-          const int nb = min(te * 8 + lr, NCE - 1);
-          const int q2b = nb / T, j0b = nb - q2b * T;
-          double d0 = 0.0, d1 = 0.0;
-#pragma unroll
-          for (int s = 0; s < KS_N; ++s) dmma(d0, d1, fPt[s], Wr[Dm::O_YE + j0b * N2 + q2b * N + min(4 * s + lc, N - 1)]);
-#pragma unroll
-          for (int i = 0; i < 2; ++i) {
-            const int n = te * 8 + 2 * lc + i;
-            if (lr < T && n < NCE) {
-              const int q2 = n / T, j0 = n - q2 * T;
-              Wr[Dm::O_ZE + q2 * T2 + lr * T + j0] = i ? d1 : d0;
-            }
+            if (n < P2) a.Fz1[(z * 3 + c) * P3 + lr * P2 + n] = d[t][i];
           }
         }
       }
-    }
-    kw_bar();
-    {   // A^T -> global
-      constexpr int NTL = (P2 + 7) / 8, NTE = (T2 + 7) / 8;
-      for (int j = kwarp; j < 3 * NTL + NTE; j += NKWW) {
-        if (j < 3 * NTL) {
-          const int c = j / NTL, tl = j - c * NTL;
-          const int nb = min(tl * 8 + lr, P2 - 1);
-          const double *Zb = Wr + Dm::O_Z + c * 2 * N * P2 + nb;
-          double d0 = 0.0, d1 = 0.0;
+      constexpr int NTE = (T2 + 7) / 8;
+      for (int te = kwarp; te < NTE; te += NKWW) {
+        const int nb = min(te * 8 + lr, T2 - 1);
+        double d0 = 0.0, d1 = 0.0;
 #pragma unroll
-          for (int s = 0; s < KS_N; ++s) {
-            const int q2 = min(4 * s + lc, N - 1);
-            dmma(d0, d1, fBt[s], Zb[q2 * P2]);
-            dmma(d0, d1, fGt[s], Zb[(N + q2) * P2]);
-          }
-          if (lr < P) {
+        for (int s = 0; s < KS_N; ++s) dmma(d0, d1, fPt[s], Wr[Dm::O_ZE + min(4 * s + lc, N - 1) * T2 + nb]);
+        if (lr < T) {
 #pragma unroll
-            for (int i = 0; i < 2; ++i) {
-              const int n = tl * 8 + 2 * lc + i;
-              if (n < P2) a.Fz1[(z * 3 + c) * P3 + lr * P2 + n] = i ? d1 : d0;
-            }
-          }
-        } else {
-          const int te = j - 3 * NTL;
-          const int nb = min(te * 8 + lr, T2 - 1);
-          double d0 = 0.0, d1 = 0.0;
-#pragma unroll
-          for (int s = 0; s < KS_N; ++s) dmma(d0, d1, fPt[s], Wr[Dm::O_ZE + min(4 * s + lc, N - 1) * T2 + nb]);
-          if (lr < T) {
-#pragma unroll
-            for (int i = 0; i < 2; ++i) {
-              const int n = te * 8 + 2 * lc + i;
-              if (n < T2) a.FTv[z * T3 + lr * T2 + n] = i ? d1 : d0;
-            }
+          for (int i = 0; i < 2; ++i) {
+            const int n = te * 8 + 2 * lc + i;
+            if (n < T2) a.FTv[z * T3 + lr * T2 + n] = i ? d1 : d0;
           }
         }
       }
