@@ -97,15 +97,15 @@ KB1Variant variant3v3() {
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3v3<K, ZPC, MINB>, (const void *)&kb1_v3_3d<K, ZPC, MINB>,
                     false};
 }
-template <int K>
+template <int K, int MODE>
 void launch3v4(const KB1Args &a, int grid, cudaStream_t s) {
-  using C = KB1V4Cfg<K>;
-  kb1_v4_3d<K><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+  using C = KB1V4Cfg<K, MODE>;
+  kb1_v4_3d<K, MODE><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
 }
-template <int K>
+template <int K, int MODE>
 KB1Variant variant3v4() {
-  using C = KB1V4Cfg<K>;
-  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v4<K>, (const void *)&kb1_v4_3d<K>, true};
+  using C = KB1V4Cfg<K, MODE>;
+  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v4<K, MODE>, (const void *)&kb1_v4_3d<K, MODE>, true};
 }
 template <int K, int ZPC, int MINB>
 KB1Variant variant3() {
@@ -130,9 +130,10 @@ KB1Variant select_variant(int dim, int k) {
       case 4: return variant3<4, 4, 2>();
     }
   }
+  if (dim == 3 && force && strcmp(force, "v4m1") == 0 && k == 4) return variant3v4<4, 1>();
   if (dim == 3 && !force) {
     switch (k) {
-      case 4: return variant3v4<4>();
+      case 4: return variant3v4<4, 0>();
     }
   }
   if (dim == 3 && !(force && strcmp(force, "v2") == 0)) {

@@ -39,14 +39,21 @@ struct V4Dims {
   static constexpr int MT = (N + 7) / 8, KS_P = (P + 3) / 4, KS_N = (N + 3) / 4, KS_T = (T + 3) / 4;
 };
 
-template <int K>
+// MODE 0: 2 points per point-thread (Nq/2 threads, 168 registers) + 8 DMMA warps (88 registers)
+// MODE 1: 1 point per point-thread (Nq threads, 104 registers)    + 4 DMMA warps (64 registers)
+// setmaxnreg only redistributes the CTA's launch allocation (NTH x floor8(65536 / NTH) registers).
+template <int K, int MODE>
 struct KB1V4Cfg {
   using Dm = V4Dims<K>;
-  static constexpr int NPW = (Dm::TPZ + 127) / 128 * 128;  // point warps' threads (whole warpgroups)
-  static constexpr int NKW = 256;                          // contraction warps' threads (2 warpgroups)
+  static constexpr int QPT = MODE == 0 ? 2 : 1;                           // points per point-thread
+  static constexpr int NPW = (Dm::N3 / QPT + 127) / 128 * 128;            // whole warpgroups
+  static constexpr int NKW = MODE == 0 ? 256 : 128;
   static constexpr int NTH = NPW + NKW;
   // register split by setmaxnreg (the launch gives 65536 / NTH): point warps get more, DMMA warps less
-  static constexpr int REG_PW = NTH == 512 ? 168 : 232, REG_KW = NTH == 512 ? 88 : 56;
+  static constexpr int REG_PW = MODE == 0 ? 168 : 104, REG_KW = MODE == 0 ? 88 : 64;
+  static constexpr int KWCH = MODE == 0 ? 8 : 2;                          // DMMA tiles in flight per warp
+  static constexpr int REG_LAUNCH = (65536 / NTH) / 8 * 8;
+  static_assert(NPW * REG_PW + NKW * REG_KW <= NTH * REG_LAUNCH, "register split exceeds the CTA's allocation");
   static constexpr int SMEM_BYTES = Dm::TOTAL * 8;
 };
 
@@ -58,16 +65,18 @@ __device__ __forceinline__ int opaque_tid() {
   return t;
 }
 
-__device__ __forceinline__ void kw_bar() { asm volatile("bar.sync 1, 256;\n" ::: "memory"); }
+template <int NKW>
+__device__ __forceinline__ void kw_bar() { asm volatile("bar.sync 1, %0;\n" ::"n"(NKW) : "memory"); }
 
-template <int K>
-__global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a) {
+template <int K, int MODE>
+__global__ void __launch_bounds__(KB1V4Cfg<K, MODE>::NTH, 1) kb1_v4_3d(const KB1Args a) {
   using Dm = V4Dims<K>;
-  using Cfg = KB1V4Cfg<K>;
+  using Cfg = KB1V4Cfg<K, MODE>;
   constexpr int N = Dm::N, P = Dm::P, T = Dm::T, P2 = Dm::P2, P3 = Dm::P3, T2 = Dm::T2, T3 = Dm::T3;
   constexpr int N2 = Dm::N2, N3 = Dm::N3, NH = Dm::NH, TPZ = Dm::TPZ;
   constexpr int KS_P = Dm::KS_P, KS_N = Dm::KS_N, KS_T = Dm::KS_T;
-  constexpr int NPW = Cfg::NPW, NKW = Cfg::NKW, NKWW = NKW / 32;
+  constexpr int NPW = Cfg::NPW, NKW = Cfg::NKW, NKWW = NKW / 32, KWCH = Cfg::KWCH;
+  static_assert(NKW >= P3, "the gather gives one node per DMMA-warp thread");
   static_assert(Dm::MT == 1, "kb1_v4: rows in one block of 8 (k <= 4)");
   extern __shared__ double smem[];
   double *sTab = smem;
@@ -124,35 +133,37 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
     if (ktid < 10) js[ktid] = sXE[Dm::XE_J + ktid];
     double *Tr = sWk;
     {   // stage A: each warp takes tiles kwarp, kwarp + 8, ... of the 6 P^2 columns at once (loads first)
-      constexpr int NC = 6 * P2, NTL = (NC + 7) / 8, JPW = (NTL + NKWW - 1) / NKWW;
-      double bx[JPW][KS_P];
-#pragma unroll
-      for (int t = 0; t < JPW; ++t) {
-        const int nb = min((kwarp + t * NKWW) * 8 + lr, NC - 1);
-        const int fb = nb / P2, ab_ = nb - fb * P2;
-#pragma unroll
-        for (int s = 0; s < KS_P; ++s) bx[t][s] = sXE[Dm::XE_X + fb * P3 + min(4 * s + lc, P - 1) * P2 + ab_];
-      }
-      double db[JPW][2], dg[JPW][2];
-#pragma unroll
-      for (int t = 0; t < JPW; ++t) {
-        db[t][0] = db[t][1] = dg[t][0] = dg[t][1] = 0.0;
-#pragma unroll
-        for (int s = 0; s < KS_P; ++s) {
-          dmma(db[t][0], db[t][1], fB[s], bx[t][s]);
-          dmma(dg[t][0], dg[t][1], fG[s], bx[t][s]);
+      constexpr int NC = 6 * P2, NTL = (NC + 7) / 8, JPWT = (NTL + NKWW - 1) / NKWW, JPW = JPWT < KWCH ? JPWT : KWCH;
+      for (int t0 = 0; t0 < JPWT; t0 += JPW) {
+        double bx[JPW][KS_P];
+  #pragma unroll
+        for (int t = 0; t < JPW; ++t) {
+          const int nb = min((kwarp + (t0 + t) * NKWW) * 8 + lr, NC - 1);
+          const int fb = nb / P2, ab_ = nb - fb * P2;
+  #pragma unroll
+          for (int s = 0; s < KS_P; ++s) bx[t][s] = sXE[Dm::XE_X + fb * P3 + min(4 * s + lc, P - 1) * P2 + ab_];
         }
-      }
-#pragma unroll
-      for (int t = 0; t < JPW; ++t) {
-        const int j = kwarp + t * NKWW;
-#pragma unroll
-        for (int i = 0; i < 2; ++i) {
-          const int n = j * 8 + 2 * lc + i;
-          if (j < NTL && lr < N && n < NC) {
-            const int f = n / P2, aa = n - f * P2;
-            Tr[Dm::O_T + (f * 2 + 0) * N * P2 + lr * P2 + aa] = db[t][i];
-            Tr[Dm::O_T + (f * 2 + 1) * N * P2 + lr * P2 + aa] = dg[t][i];
+        double db[JPW][2], dg[JPW][2];
+  #pragma unroll
+        for (int t = 0; t < JPW; ++t) {
+          db[t][0] = db[t][1] = dg[t][0] = dg[t][1] = 0.0;
+  #pragma unroll
+          for (int s = 0; s < KS_P; ++s) {
+            dmma(db[t][0], db[t][1], fB[s], bx[t][s]);
+            dmma(dg[t][0], dg[t][1], fG[s], bx[t][s]);
+          }
+        }
+  #pragma unroll
+        for (int t = 0; t < JPW; ++t) {
+          const int j = kwarp + (t0 + t) * NKWW;
+  #pragma unroll
+          for (int i = 0; i < 2; ++i) {
+            const int n = j * 8 + 2 * lc + i;
+            if (j < NTL && lr < N && n < NC) {
+              const int f = n / P2, aa = n - f * P2;
+              Tr[Dm::O_T + (f * 2 + 0) * N * P2 + lr * P2 + aa] = db[t][i];
+              Tr[Dm::O_T + (f * 2 + 1) * N * P2 + lr * P2 + aa] = dg[t][i];
+            }
           }
         }
       }
@@ -169,46 +180,48 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
         }
       }
     }
-    kw_bar();
+    kw_bar<NKW>();
     {   // stage B: U0 = B.TB, U1 = G.TB, U2 = B.TG; tiles kwarp, kwarp + 8, ... at once
-      constexpr int NC = 6 * N * P, NTL = (NC + 7) / 8, JPW = (NTL + NKWW - 1) / NKWW;
-      double tb[JPW][KS_P], tg[JPW][KS_P];
-#pragma unroll
-      for (int t = 0; t < JPW; ++t) {
-        const int nb = min((kwarp + t * NKWW) * 8 + lr, NC - 1);
-        const int fb = nb / (N * P), rb = nb - fb * (N * P), q2b = rb / P, a0b = rb - q2b * P;
-        const double *TBb = Tr + Dm::O_T + ((fb * 2 + 0) * N + q2b) * P2 + a0b;
-#pragma unroll
-        for (int s = 0; s < KS_P; ++s) {
-          const int a1 = min(4 * s + lc, P - 1);
-          tb[t][s] = TBb[a1 * P];
-          tg[t][s] = TBb[N * P2 + a1 * P];
+      constexpr int NC = 6 * N * P, NTL = (NC + 7) / 8, JPWT = (NTL + NKWW - 1) / NKWW, JPW = JPWT < KWCH ? JPWT : KWCH;
+      for (int t0 = 0; t0 < JPWT; t0 += JPW) {
+        double tb[JPW][KS_P], tg[JPW][KS_P];
+  #pragma unroll
+        for (int t = 0; t < JPW; ++t) {
+          const int nb = min((kwarp + (t0 + t) * NKWW) * 8 + lr, NC - 1);
+          const int fb = nb / (N * P), rb = nb - fb * (N * P), q2b = rb / P, a0b = rb - q2b * P;
+          const double *TBb = Tr + Dm::O_T + ((fb * 2 + 0) * N + q2b) * P2 + a0b;
+  #pragma unroll
+          for (int s = 0; s < KS_P; ++s) {
+            const int a1 = min(4 * s + lc, P - 1);
+            tb[t][s] = TBb[a1 * P];
+            tg[t][s] = TBb[N * P2 + a1 * P];
+          }
         }
-      }
-      double u[JPW][3][2];
-#pragma unroll
-      for (int t = 0; t < JPW; ++t) {
-#pragma unroll
-        for (int m = 0; m < 3; ++m) u[t][m][0] = u[t][m][1] = 0.0;
-#pragma unroll
-        for (int s = 0; s < KS_P; ++s) {
-          dmma(u[t][0][0], u[t][0][1], fB[s], tb[t][s]);
-          dmma(u[t][1][0], u[t][1][1], fG[s], tb[t][s]);
-          dmma(u[t][2][0], u[t][2][1], fB[s], tg[t][s]);
+        double u[JPW][3][2];
+  #pragma unroll
+        for (int t = 0; t < JPW; ++t) {
+  #pragma unroll
+          for (int m = 0; m < 3; ++m) u[t][m][0] = u[t][m][1] = 0.0;
+  #pragma unroll
+          for (int s = 0; s < KS_P; ++s) {
+            dmma(u[t][0][0], u[t][0][1], fB[s], tb[t][s]);
+            dmma(u[t][1][0], u[t][1][1], fG[s], tb[t][s]);
+            dmma(u[t][2][0], u[t][2][1], fB[s], tg[t][s]);
+          }
         }
-      }
-#pragma unroll
-      for (int t = 0; t < JPW; ++t) {
-        const int j = kwarp + t * NKWW;
-#pragma unroll
-        for (int i = 0; i < 2; ++i) {
-          const int n = j * 8 + 2 * lc + i;
-          if (j < NTL && lr < N && n < NC) {
-            const int f = n / (N * P), rr = n - f * (N * P), q2 = rr / P, a0 = rr - q2 * P;
-            double *U = ub + (((f * 3) * N + q2) * N + lr) * P + a0;
-            U[0] = u[t][0][i];
-            U[N2 * P] = u[t][1][i];
-            U[2 * N2 * P] = u[t][2][i];
+  #pragma unroll
+        for (int t = 0; t < JPW; ++t) {
+          const int j = kwarp + (t0 + t) * NKWW;
+  #pragma unroll
+          for (int i = 0; i < 2; ++i) {
+            const int n = j * 8 + 2 * lc + i;
+            if (j < NTL && lr < N && n < NC) {
+              const int f = n / (N * P), rr = n - f * (N * P), q2 = rr / P, a0 = rr - q2 * P;
+              double *U = ub + (((f * 3) * N + q2) * N + lr) * P + a0;
+              U[0] = u[t][0][i];
+              U[N2 * P] = u[t][1][i];
+              U[2 * N2 * P] = u[t][2][i];
+            }
           }
         }
       }
@@ -276,47 +289,49 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
         }
       }
     }
-    kw_bar();
+    kw_bar<NKW>();
     {   // B^T: jobs (c, tile) spread over the warps, each warp's jobs loaded/multiplied/stored together
-      constexpr int NC = N * P, NTL = (NC + 7) / 8, NJ = 3 * NTL, JPW = (NJ + NKWW - 1) / NKWW;
-      double y[JPW][3][KS_N];
-#pragma unroll
-      for (int t = 0; t < JPW; ++t) {
-        const int j = min(kwarp + t * NKWW, NJ - 1);
-        const int c = j / NTL, tl = j - c * NTL;
-        const int nb = min(tl * 8 + lr, NC - 1);
-        const int q2b = nb / P, a0b = nb - q2b * P;
-        const double *Yb = Wr + Dm::O_Y + (c * 3 * P + a0b) * N2 + q2b * N;
-#pragma unroll
-        for (int s = 0; s < KS_N; ++s) {
-          const int q1 = min(4 * s + lc, N - 1);
-          y[t][0][s] = Yb[q1];
-          y[t][1][s] = Yb[P * N2 + q1];
-          y[t][2][s] = Yb[2 * P * N2 + q1];
+      constexpr int NC = N * P, NTL = (NC + 7) / 8, NJ = 3 * NTL, JPWT = (NJ + NKWW - 1) / NKWW, JPW = JPWT < KWCH ? JPWT : KWCH;
+      for (int t0 = 0; t0 < JPWT; t0 += JPW) {
+        double y[JPW][3][KS_N];
+  #pragma unroll
+        for (int t = 0; t < JPW; ++t) {
+          const int j = min(kwarp + (t0 + t) * NKWW, NJ - 1);
+          const int c = j / NTL, tl = j - c * NTL;
+          const int nb = min(tl * 8 + lr, NC - 1);
+          const int q2b = nb / P, a0b = nb - q2b * P;
+          const double *Yb = Wr + Dm::O_Y + (c * 3 * P + a0b) * N2 + q2b * N;
+  #pragma unroll
+          for (int s = 0; s < KS_N; ++s) {
+            const int q1 = min(4 * s + lc, N - 1);
+            y[t][0][s] = Yb[q1];
+            y[t][1][s] = Yb[P * N2 + q1];
+            y[t][2][s] = Yb[2 * P * N2 + q1];
+          }
         }
-      }
-      double zb[JPW][2], zg[JPW][2];
-#pragma unroll
-      for (int t = 0; t < JPW; ++t) {
-        zb[t][0] = zb[t][1] = zg[t][0] = zg[t][1] = 0.0;
-#pragma unroll
-        for (int s = 0; s < KS_N; ++s) {
-          dmma(zb[t][0], zb[t][1], fBt[s], y[t][0][s]);
-          dmma(zb[t][0], zb[t][1], fGt[s], y[t][1][s]);
-          dmma(zg[t][0], zg[t][1], fBt[s], y[t][2][s]);
+        double zb[JPW][2], zg[JPW][2];
+  #pragma unroll
+        for (int t = 0; t < JPW; ++t) {
+          zb[t][0] = zb[t][1] = zg[t][0] = zg[t][1] = 0.0;
+  #pragma unroll
+          for (int s = 0; s < KS_N; ++s) {
+            dmma(zb[t][0], zb[t][1], fBt[s], y[t][0][s]);
+            dmma(zb[t][0], zb[t][1], fGt[s], y[t][1][s]);
+            dmma(zg[t][0], zg[t][1], fBt[s], y[t][2][s]);
+          }
         }
-      }
-#pragma unroll
-      for (int t = 0; t < JPW; ++t) {
-        const int j = kwarp + t * NKWW;
-        const int c = j / NTL, tl = j - c * NTL;
-#pragma unroll
-        for (int i = 0; i < 2; ++i) {
-          const int n = tl * 8 + 2 * lc + i;
-          if (j < NJ && lr < P && n < NC) {
-            const int q2 = n / P, a0 = n - q2 * P;
-            Wr[Dm::O_Z + ((c * 2 + 0) * N + q2) * P2 + lr * P + a0] = zb[t][i];
-            Wr[Dm::O_Z + ((c * 2 + 1) * N + q2) * P2 + lr * P + a0] = zg[t][i];
+  #pragma unroll
+        for (int t = 0; t < JPW; ++t) {
+          const int j = kwarp + (t0 + t) * NKWW;
+          const int c = j / NTL, tl = j - c * NTL;
+  #pragma unroll
+          for (int i = 0; i < 2; ++i) {
+            const int n = tl * 8 + 2 * lc + i;
+            if (j < NJ && lr < P && n < NC) {
+              const int q2 = n / P, a0 = n - q2 * P;
+              Wr[Dm::O_Z + ((c * 2 + 0) * N + q2) * P2 + lr * P + a0] = zb[t][i];
+              Wr[Dm::O_Z + ((c * 2 + 1) * N + q2) * P2 + lr * P + a0] = zg[t][i];
+            }
           }
         }
       }
@@ -337,42 +352,44 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
         }
       }
     }
-    kw_bar();
+    kw_bar<NKW>();
     {   // A^T -> global: jobs (c, tile) and the F^T v tiles, each warp's jobs loaded/multiplied/stored together
-      constexpr int NTL = (P2 + 7) / 8, NJ = 3 * NTL, JPW = (NJ + NKWW - 1) / NKWW;
-      double zv[JPW][2][KS_N];
-#pragma unroll
-      for (int t = 0; t < JPW; ++t) {
-        const int j = min(kwarp + t * NKWW, NJ - 1);
-        const int c = j / NTL, tl = j - c * NTL;
-        const int nb = min(tl * 8 + lr, P2 - 1);
-        const double *Zb = Wr + Dm::O_Z + c * 2 * N * P2 + nb;
-#pragma unroll
-        for (int s = 0; s < KS_N; ++s) {
-          const int q2 = min(4 * s + lc, N - 1);
-          zv[t][0][s] = Zb[q2 * P2];
-          zv[t][1][s] = Zb[(N + q2) * P2];
+      constexpr int NTL = (P2 + 7) / 8, NJ = 3 * NTL, JPWT = (NJ + NKWW - 1) / NKWW, JPW = JPWT < KWCH ? JPWT : KWCH;
+      for (int t0 = 0; t0 < JPWT; t0 += JPW) {
+        double zv[JPW][2][KS_N];
+  #pragma unroll
+        for (int t = 0; t < JPW; ++t) {
+          const int j = min(kwarp + (t0 + t) * NKWW, NJ - 1);
+          const int c = j / NTL, tl = j - c * NTL;
+          const int nb = min(tl * 8 + lr, P2 - 1);
+          const double *Zb = Wr + Dm::O_Z + c * 2 * N * P2 + nb;
+  #pragma unroll
+          for (int s = 0; s < KS_N; ++s) {
+            const int q2 = min(4 * s + lc, N - 1);
+            zv[t][0][s] = Zb[q2 * P2];
+            zv[t][1][s] = Zb[(N + q2) * P2];
+          }
         }
-      }
-      double d[JPW][2];
-#pragma unroll
-      for (int t = 0; t < JPW; ++t) {
-        d[t][0] = d[t][1] = 0.0;
-#pragma unroll
-        for (int s = 0; s < KS_N; ++s) {
-          dmma(d[t][0], d[t][1], fBt[s], zv[t][0][s]);
-          dmma(d[t][0], d[t][1], fGt[s], zv[t][1][s]);
+        double d[JPW][2];
+  #pragma unroll
+        for (int t = 0; t < JPW; ++t) {
+          d[t][0] = d[t][1] = 0.0;
+  #pragma unroll
+          for (int s = 0; s < KS_N; ++s) {
+            dmma(d[t][0], d[t][1], fBt[s], zv[t][0][s]);
+            dmma(d[t][0], d[t][1], fGt[s], zv[t][1][s]);
+          }
         }
-      }
-#pragma unroll
-      for (int t = 0; t < JPW; ++t) {
-        const int j = kwarp + t * NKWW;
-        const int c = j / NTL, tl = j - c * NTL;
-        if (j < NJ && lr < P) {
-#pragma unroll
-          for (int i = 0; i < 2; ++i) {
-            const int n = tl * 8 + 2 * lc + i;
-            if (n < P2) a.Fz1[(z * 3 + c) * P3 + lr * P2 + n] = d[t][i];
+  #pragma unroll
+        for (int t = 0; t < JPW; ++t) {
+          const int j = kwarp + (t0 + t) * NKWW;
+          const int c = j / NTL, tl = j - c * NTL;
+          if (j < NJ && lr < P) {
+  #pragma unroll
+            for (int i = 0; i < 2; ++i) {
+              const int n = tl * 8 + 2 * lc + i;
+              if (n < P2) a.Fz1[(z * 3 + c) * P3 + lr * P2 + n] = d[t][i];
+            }
           }
         }
       }
@@ -391,7 +408,7 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
         }
       }
     }
-    kw_bar();   // Y/Z scratch free again (stage A of the next forward pass overwrites it)
+    kw_bar<NKW>();   // Y/Z scratch free again (stage A of the next forward pass overwrites it)
   };
 
   // ---------------- PW: stage C + point evaluation of zone z from U buffer ub into S buffer sb ----------
@@ -456,6 +473,44 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
     bad |= oa.bad | ob.bad;
   };
 
+  auto pw_point1 = [&](const double *ub, const double *js, double *sb, int64_t z) {
+    // one point per thread: q = tid
+    const int q0 = tid % N, q1s = (tid / N) % N, q2s = tid / N2;
+    const int q = tid;
+    const double R = __ldg(a.rho0detJ0 + z * N3 + q);
+    double g[18];
+#pragma unroll
+    for (int i = 0; i < 18; ++i) g[i] = 0.0;
+#pragma unroll
+    for (int a0 = 0; a0 < P; ++a0) {
+      const double b = tB[q0 * P + a0], gg = tG[q0 * P + a0];
+#pragma unroll
+      for (int f = 0; f < 6; ++f)
+#pragma unroll
+        for (int m = 0; m < 3; ++m)
+          g[f * 3 + m] = fma(m == 0 ? gg : b, ub[(((f * 3 + m) * N + q2s) * N + q1s) * P + a0], g[f * 3 + m]);
+    }
+    double eq = 0.0;
+#pragma unroll
+    for (int j0 = 0; j0 < T; ++j0) eq = fma(tPhi[q0 * T + j0], ub[Dm::O_UE + (q2s * N + q1s) * T + j0], eq);
+    double Jm[3][3], Gv[3][3];
+#pragma unroll
+    for (int c = 0; c < 3; ++c)
+#pragma unroll
+      for (int d = 0; d < 3; ++d) { Jm[c][d] = g[c * 3 + d]; Gv[c][d] = g[9 + c * 3 + d]; }
+    PointOut<3> o;
+    point_eval3(Jm, Gv, eq, R, sW[q0] * sW[q1s] * sW[q2s], js[9], js, a.ph, o);
+#pragma unroll
+    for (int cd = 0; cd < 9; ++cd) sb[cd * N3 + q] = o.S[cd / 3][cd % 3];
+    sb[Dm::O_PQ + q] = o.P;
+    if (a.Sq != nullptr) {
+#pragma unroll
+      for (int cd = 0; cd < 9; ++cd) a.Sq[(z * N3 + q) * 9 + cd] = o.S[cd / 3][cd % 3];
+    }
+    dtmin = fmin(dtmin, o.dt);
+    bad |= o.bad;
+  };
+
   // ---------------- the two groups run separate code paths from here on (register split) ----------------
   // Both execute the same number of CTA barriers (bar 0): 1 after the prologue + (nz + 1) in the loop.
   if (is_kw) {
@@ -464,7 +519,7 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
     kw_issue(0);
     kw_load_id(1);
     cp_async_wait<0>();
-    kw_bar();
+    kw_bar<NKW>();
     if (nz > 0) kw_forward(sU, sJ);
     __syncthreads();
     long long t_work = 0;
@@ -474,7 +529,7 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
       kw_load_id(i + 2);
       if (i >= 1) kw_back(sS + ((i - 1) & 1) * Dm::SBUF, zone_of(i - 1));
       cp_async_wait<0>();
-      kw_bar();
+      kw_bar<NKW>();
       if (i + 1 < nz) kw_forward(sU + ((i + 1) & 1) * Dm::UBUF, sJ + ((i + 1) & 1) * 10);
       t_work += clock64() - t0;
       __syncthreads();
@@ -487,7 +542,11 @@ __global__ void __launch_bounds__(KB1V4Cfg<K>::NTH, 1) kb1_v4_3d(const KB1Args a
   long long t_work = 0, t_all = clock64();
   for (int64_t i = 0; i <= nz; ++i) {
     const long long t0 = clock64();
-    if (i < nz && tid < TPZ) pw_point(sU + (i & 1) * Dm::UBUF, sJ + (i & 1) * 10, sS + (i & 1) * Dm::SBUF, zone_of(i));
+    if (MODE == 0) {
+      if (i < nz && tid < TPZ) pw_point(sU + (i & 1) * Dm::UBUF, sJ + (i & 1) * 10, sS + (i & 1) * Dm::SBUF, zone_of(i));
+    } else {
+      if (i < nz && tid < N3) pw_point1(sU + (i & 1) * Dm::UBUF, sJ + (i & 1) * 10, sS + (i & 1) * Dm::SBUF, zone_of(i));
+    }
     t_work += clock64() - t0;
     __syncthreads();
   }
