@@ -197,3 +197,25 @@ def sampled_parity(orc, name, which, n_nodes=48, n_zones=48, seed=0):
                                         ("C5", "S1")])
 def test_full_size_sampled(orc, name, which):
     sampled_parity(orc, name, which, n_nodes=24 if name == "C5" else 48, n_zones=8 if name == "C5" else 48)
+
+
+def test_non_affine_initial_mesh(orc):
+    """Reading R19: the GPU keeps J0^{-1} per zone, so a curved initial mesh is rejected when the
+    viscosity (which needs J0) is on, and evaluated normally when it is off."""
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    _torch()
+    m, s = synth.config("C3", "S1", N=(3, 3, 3))
+    curved = synth.Mesh(m.dim, m.order, m.N, m.L, s.x.copy(), m.zone_nodes, m.zone_mat, m.mat_gamma)
+    with pytest.raises(cf.BlastCFError) as ei:
+        cf.from_synth(curved)
+    assert ei.value.code == cf.EUNSUPPORTED
+    gp = cf.default_params()
+    gp.use_viscosity = 0
+    check(curved, s, orc, oparams=orc.Params(use_viscosity=0), gparams=gp)
+
+
+def test_multi_material_gamma(orc):
+    """Per-zone gamma through zone_mat / mat_gamma (triple point, 3 materials)."""
+    m, s = synth.config("C5", "S1", N=(6, 3, 3), k=2)
+    assert len(np.unique(m.zone_mat)) == 3
+    check(m, s, orc)
