@@ -92,6 +92,29 @@ class ClockSampler:
         return {"sm_mhz": statistics.median(sm), "sm_max_mhz": smax, "reasons": sorted(reasons), "samples": len(sm)}
 
 
+class EnergyMeter:
+    """NVML total-energy counter around the timed region (the paper's energy theme,
+    PAPER.md:906-1120).  Reports J per step and uJ per zone; None if NVML is unavailable."""
+
+    def __init__(self, gpu_index):
+        self.h = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(gpu_index)
+        except Exception:
+            self.h = None
+
+    def read_mj(self):
+        if self.h is None:
+            return None
+        try:
+            return self.nv.nvmlDeviceGetTotalEnergyConsumption(self.h)
+        except Exception:
+            return None
+
+
 def workload_desc(name):
     import synth
     c = synth.CONFIGS[name]
@@ -210,11 +233,14 @@ def run_ours(args):
             if time.perf_counter() - t_w > 0.4:
                 break
         barrier()
+        meter = EnergyMeter(local if world > 1 else 0)
+        e_start = meter.read_mj()
         ev0.record(stream)
         for _ in range(args.steps):
             h.eval(x, v, e, r, out=out)
         ev1.record(stream)
         barrier()
+        e_end = meter.read_mj()
     ms = ev0.elapsed_time(ev1)
     if world > 1:
         tt = torch.tensor([ms], device=dev, dtype=torch.float64)
@@ -271,6 +297,11 @@ def run_ours(args):
                "sample": f"first {nz} of {Zg} zones of the same C4 S1 state, one evaluation (plain C oracle, "
                          f"OpenMP over zones, serial assembly), {tc:.1f} s"}
 
+    energy = None
+    if e_start is not None and e_end is not None and e_end > e_start:
+        joules = (e_end - e_start) / 1e3
+        energy = {"joules_per_step": joules / args.steps, "uJ_per_zone": 1e6 * joules / args.steps / Zg,
+                  "avg_power_w": joules / (ms / 1e3), "source": "NVML total energy counter, rank 0's GPU"}
     if rank == 0:
         clocks = clk.summary()
         line = {
@@ -292,6 +323,7 @@ def run_ours(args):
                          "traffic_source": tsrc},
             "e2e": e2e,
             "gpu_launches": int(info["kernels_per_eval"] * args.steps),
+            "energy": energy,
             "clocks": clocks,
             "cpu_baseline": cpu,
             "launch": {k: info[k] for k in ("zones_per_cta", "threads_per_cta", "num_ctas", "smem_bytes",

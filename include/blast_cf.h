@@ -124,6 +124,19 @@ int blast_cf_eval_loopback(blast_cf *const *hs, int n, const double *const *x, c
                            const double *const *e, const double *const *rho0detJ0, double *const *out_Fdot1,
                            double *const *out_FTv, double *const *out_dt_min);
 
+/* Order-adaptive kernel selection (the paper's autotuning, §3.2.1, done at the
+ * caller's request instead of over sampling periods): times every candidate corner-force kernel for the
+ * handle's (dim, k) — e.g. for 3D k = 4 the warp-specialized pipeline (two register splits), the
+ * CTA-synchronous DMMA kernel, the DFMA kernel and the per-slab kernel — on the given device inputs,
+ * `reps` evaluations each, and keeps the fastest for all later evals.  ms_out[capacity] receives the
+ * per-candidate milliseconds in candidate order, *num_candidates their count; outputs are overwritten
+ * as by blast_cf_eval.  Synchronous.  blast_cf_variant_name(h, i) names candidate i (i < 0: the one
+ * in use); the BLAST_CF_KB1 environment variable (a name) overrides the default at create. */
+int blast_cf_autotune(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                      double *out_Fdot1, double *out_FTv, double *out_dt_min, int reps, double *ms_out, int capacity,
+                      int *num_candidates);
+const char *blast_cf_variant_name(const blast_cf *h, int index);
+
 typedef struct {
   int32_t dim, order, nq, nk, nt;
   int64_t num_zones, num_nodes;

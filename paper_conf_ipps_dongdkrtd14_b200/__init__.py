@@ -95,10 +95,13 @@ def lib():
     L.blast_cf_debug_cta_dt.argtypes = [vp, vp, i64, ctypes.POINTER(i32), ctypes.POINTER(i32)]
     L.blast_cf_debug_stage_clocks.argtypes = [vp, vp, i64]
     L.blast_cf_eval_loopback.argtypes = [vp, ctypes.c_int, vp, vp, vp, vp, vp, vp, vp]
+    L.blast_cf_autotune.argtypes = [vp] * 8 + [ctypes.c_int, vp, ctypes.c_int, ctypes.POINTER(ctypes.c_int)]
+    L.blast_cf_variant_name.argtypes = [vp, ctypes.c_int]
+    L.blast_cf_variant_name.restype = ctypes.c_char_p
     for f in ("blast_cf_create", "blast_cf_eval", "blast_cf_eval_host", "blast_cf_eval_debug_Fz", "blast_cf_get_info",
               "blast_cf_set_timing", "blast_cf_kernel_times", "blast_cf_destroy", "blast_cf_nccl_unique_id_size",
               "blast_cf_nccl_get_unique_id", "blast_cf_exchange_plan", "blast_cf_debug_cta_dt",
-              "blast_cf_debug_stage_clocks", "blast_cf_eval_loopback"):
+              "blast_cf_debug_stage_clocks", "blast_cf_eval_loopback", "blast_cf_autotune"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
     return L
@@ -252,6 +255,24 @@ class CornerForce:
                                             self._dev(e, (Z, self.nt)), self._dev(rho0detJ0, (Z, self.nq)),
                                             self._dev(Fz, Fz.shape)), "blast_cf_eval_debug_Fz")
         return Fz
+
+    def autotune(self, x, v, e, rho0detJ0, reps: int = 3):
+        """Time every candidate corner-force kernel on these inputs and keep the fastest
+        (blast_cf_autotune).  Returns {variant name: ms} and sets self.variant."""
+        F1, FTv, dt = self.alloc_outputs()
+        ms = (ctypes.c_double * 16)()
+        n = ctypes.c_int(0)
+        d, nn, Z = self.dim, self.num_nodes, self.num_zones
+        _check(lib().blast_cf_autotune(self._h, self._dev(x, (d, nn)), self._dev(v, (d, nn)), self._dev(e, (Z, self.nt)),
+                                       self._dev(rho0detJ0, (Z, self.nq)), self._dev(F1, (d, nn)),
+                                       self._dev(FTv, (Z, self.nt)), self._dev(dt, (1,)), int(reps), ms, 16,
+                                       ctypes.byref(n)), "blast_cf_autotune")
+        self.info = self.get_info()
+        return {lib().blast_cf_variant_name(self._h, i).decode(): ms[i] for i in range(n.value)}
+
+    @property
+    def variant(self) -> str:
+        return lib().blast_cf_variant_name(self._h, -1).decode()
 
     def debug_cta_dt(self):
         """(per-CTA min dt of the last eval, zones per CTA) — tests only."""

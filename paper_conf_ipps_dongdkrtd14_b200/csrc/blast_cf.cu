@@ -63,6 +63,7 @@ struct KB1Variant {
   kb1_launch_fn launch;
   const void *func;
   bool persistent;   // grid = resident CTAs; CTA c runs zone batches c, c + grid, ...
+  const char *name = nullptr;
 };
 
 template <int K, int ZPC, int MINB>
@@ -84,7 +85,7 @@ template <int K, int ZPC, int MINB>
 KB1Variant variant3v2() {
   using C = KB1V2Cfg<K, ZPC>;
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3v2<K, ZPC, MINB>, (const void *)&kb1_v2_3d<K, ZPC, MINB>,
-                    true};
+                    true, nullptr};
 }
 template <int K, int ZPC, int MINB>
 void launch3v3(const KB1Args &a, int grid, cudaStream_t s) {
@@ -95,7 +96,7 @@ template <int K, int ZPC, int MINB>
 KB1Variant variant3v3() {
   using C = KB1V3Cfg<K, ZPC>;
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3v3<K, ZPC, MINB>, (const void *)&kb1_v3_3d<K, ZPC, MINB>,
-                    false};
+                    false, nullptr};
 }
 template <int K, int MODE>
 void launch3v4(const KB1Args &a, int grid, cudaStream_t s) {
@@ -105,67 +106,63 @@ void launch3v4(const KB1Args &a, int grid, cudaStream_t s) {
 template <int K, int MODE>
 KB1Variant variant3v4() {
   using C = KB1V4Cfg<K, MODE>;
-  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v4<K, MODE>, (const void *)&kb1_v4_3d<K, MODE>, true};
+  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v4<K, MODE>, (const void *)&kb1_v4_3d<K, MODE>, true, nullptr};
 }
 template <int K, int ZPC, int MINB>
 KB1Variant variant3() {
   using C = KB1Cfg3<K, ZPC>;
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3<K, ZPC, MINB>,
-                    (const void *)&kb1_corner_force_3d<K, ZPC, MINB>, false};
+                    (const void *)&kb1_corner_force_3d<K, ZPC, MINB>, false, nullptr};
 }
 template <int K, int ZPC, int MINB>
 KB1Variant variant2() {
   using C = KB1Cfg2<K, ZPC>;
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch2<K, ZPC, MINB>,
-                    (const void *)&kb1_corner_force_2d<K, ZPC, MINB>, false};
+                    (const void *)&kb1_corner_force_2d<K, ZPC, MINB>, false, nullptr};
 }
 
-KB1Variant select_variant(int dim, int k) {
-  const char *force = getenv("BLAST_CF_KB1");   // experiments only: "v1" forces the per-slab kernel
-  if (dim == 3 && force && strcmp(force, "v1") == 0) {
-    switch (k) {
-      case 1: return variant3<1, 32, 2>();
-      case 2: return variant3<2, 16, 2>();
-      case 3: return variant3<3, 8, 2>();
-      case 4: return variant3<4, 4, 2>();
-    }
-  }
-  if (dim == 3 && force && strcmp(force, "v4m1") == 0 && k == 4) return variant3v4<4, 1>();
-  if (dim == 3 && !force) {
-    switch (k) {
-      case 4: return variant3v4<4, 0>();
-    }
-  }
-  if (dim == 3 && !(force && strcmp(force, "v2") == 0)) {
-    switch (k) {
-      case 3: return variant3v3<3, 2, 2>();
-      case 4: return variant3v3<4, 1, 2>();
-    }
-  }
+// Candidate KB1 variants per (dim, k), default first (f3 of SURVEY §8: the create-time default is the
+// measured winner of round 1; blast_cf_autotune re-times all candidates on the caller's data).
+std::vector<KB1Variant> kb1_candidates(int dim, int k) {
+  std::vector<KB1Variant> v;
+  auto add = [&](KB1Variant x, const char *name) { x.name = name; v.push_back(x); };
   if (dim == 3) {
     switch (k) {
-      case 1: return variant3v2<1, 64, 2>();
-      case 2: return variant3v2<2, 4, 3>();
-      case 3: return variant3v2<3, 2, 2>();
-      case 4: return variant3v2<4, 1, 2>();
-      case 5: return variant3<5, 2, 2>();
-      case 6: return variant3<6, 2, 1>();
-      case 7: return variant3<7, 1, 2>();
-      case 8: return variant3<8, 1, 1>();
+      case 1: add(variant3v2<1, 64, 2>(), "v2.z64"); add(variant3<1, 32, 2>(), "v1.z32"); break;
+      case 2: add(variant3v2<2, 4, 3>(), "v2.z4"); add(variant3v3<2, 4, 2>(), "v3.z4"); add(variant3<2, 16, 2>(), "v1.z16"); break;
+      case 3: add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
+      case 4:
+        add(variant3v4<4, 0>(), "v4.m0"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
+        add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
+        break;
+      case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
+      case 6: add(variant3<6, 1, 2>(), "v1.z1m2"); add(variant3<6, 2, 1>(), "v1.z2"); break;
+      case 7: add(variant3<7, 1, 2>(), "v1.z1"); break;
+      case 8: add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
     }
   } else {
     switch (k) {
-      case 1: return variant2<1, 64, 2>();
-      case 2: return variant2<2, 16, 2>();
-      case 3: return variant2<3, 8, 2>();
-      case 4: return variant2<4, 4, 2>();
-      case 5: return variant2<5, 2, 2>();
-      case 6: return variant2<6, 2, 2>();
-      case 7: return variant2<7, 1, 2>();
-      case 8: return variant2<8, 1, 2>();
+      case 1: add(variant2<1, 64, 2>(), "v1-2d.z64"); break;
+      case 2: add(variant2<2, 16, 2>(), "v1-2d.z16"); break;
+      case 3: add(variant2<3, 8, 2>(), "v1-2d.z8"); break;
+      case 4: add(variant2<4, 4, 2>(), "v1-2d.z4"); break;
+      case 5: add(variant2<5, 2, 2>(), "v1-2d.z2"); break;
+      case 6: add(variant2<6, 2, 2>(), "v1-2d.z2"); break;
+      case 7: add(variant2<7, 1, 2>(), "v1-2d.z1"); break;
+      case 8: add(variant2<8, 1, 2>(), "v1-2d.z1"); break;
     }
   }
-  return KB1Variant{0, 0, 0, nullptr, nullptr, false};
+  return v;
+}
+
+KB1Variant select_variant(int dim, int k) {
+  const std::vector<KB1Variant> c = kb1_candidates(dim, k);
+  if (c.empty()) return KB1Variant{0, 0, 0, nullptr, nullptr, false, nullptr};
+  const char *force = getenv("BLAST_CF_KB1");   // experiments: pick a candidate by name
+  if (force)
+    for (const KB1Variant &x : c)
+      if (strcmp(x.name, force) == 0) return x;
+  return c[0];
 }
 
 // Debug: F_z = A_z B^T from S(q) (kernel 7 of the paper); one CTA per zone.
@@ -331,6 +328,7 @@ struct blast_cf {
   int device = 0;
   KB1Variant var{};
   int ncta = 0, regs = 0, local_bytes = 0;
+  int64_t ncta_cap = 0;
   // device memory
   double *d_tab = nullptr, *d_J0inv = nullptr, *d_gamma = nullptr, *d_Fz1 = nullptr, *d_ctadt = nullptr;
   int32_t *d_zone_nodes = nullptr, *d_ptr = nullptr, *d_ent = nullptr;
@@ -356,6 +354,26 @@ void free_handle(blast_cf *h) {
   delete h;
 }
 
+
+// make `v` the handle's KB1: shared-memory opt-in, register / local-memory info, grid size
+int apply_variant(blast_cf *h, const KB1Variant &v) {
+  if (cudaFuncSetAttribute(v.func, cudaFuncAttributeMaxDynamicSharedMemorySize, v.smem) != cudaSuccess)
+    return fail(BLAST_CF_ECUDA, "cudaFuncSetAttribute(smem=%d): %s", v.smem, cudaGetErrorString(cudaGetLastError()));
+  cudaFuncAttributes fa;
+  if (cudaFuncGetAttributes(&fa, v.func) == cudaSuccess) {
+    h->regs = fa.numRegs;
+    h->local_bytes = (int)fa.localSizeBytes;
+  }
+  h->var = v;
+  h->ncta = (int)((h->Z + v.zpc - 1) / v.zpc);
+  if (v.persistent && h->ncta > 0) {
+    int occ = 0, sms = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, v.func, v.nth, v.smem);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device);
+    h->ncta = std::min<int>(h->ncta, std::max(1, occ) * std::max(1, sms));
+  }
+  return BLAST_CF_OK;
+}
 
 int check_async(blast_cf *h) {
   cudaError_t e = cudaGetLastError();
@@ -543,21 +561,9 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
   // ---- kernel variant ----
   h->var = select_variant(dim, order);
   if (!h->var.launch) return bail(fail(BLAST_CF_EUNSUPPORTED, "no kernel for dim %d order %d", dim, order));
-  if (cudaFuncSetAttribute(h->var.func, cudaFuncAttributeMaxDynamicSharedMemorySize, h->var.smem) != cudaSuccess)
-    return bail(fail(BLAST_CF_ECUDA, "cudaFuncSetAttribute(smem=%d): %s", h->var.smem,
-                     cudaGetErrorString(cudaGetLastError())));
-  cudaFuncAttributes fa;
-  if (cudaFuncGetAttributes(&fa, h->var.func) == cudaSuccess) {
-    h->regs = fa.numRegs;
-    h->local_bytes = (int)fa.localSizeBytes;
-  }
-  h->ncta = (int)((Z + h->var.zpc - 1) / h->var.zpc);
-  if (h->var.persistent && h->ncta > 0) {
-    int occ = 0, sms = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, h->var.func, h->var.nth, h->var.smem);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device);
-    h->ncta = std::min<int>(h->ncta, std::max(1, occ) * std::max(1, sms));
-  }
+  if ((rc = apply_variant(h, h->var))) return bail(rc);
+  for (const KB1Variant &c : kb1_candidates(dim, order))   // per-CTA dt slots for any candidate
+    h->ncta_cap = std::max<int64_t>(h->ncta_cap, (Z + c.zpc - 1) / c.zpc);
 
   // ---- uploads ----
   if ((rc = upload(&h->d_tab, tab.data(), tab.size())) ||
@@ -567,11 +573,11 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
       (rc = upload(&h->d_ptr, ptr.data(), ptr.size())) || (rc = upload(&h->d_ent, ent.data(), ent.size())))
     return bail(rc);
   if (cudaMalloc(&h->d_Fz1, std::max<size_t>((size_t)Z * dim * nk, 1) * sizeof(double)) != cudaSuccess ||
-      cudaMalloc(&h->d_ctadt, std::max(h->ncta, 1) * sizeof(double)) != cudaSuccess)
+      cudaMalloc(&h->d_ctadt, std::max<int64_t>(h->ncta_cap, 1) * sizeof(double)) != cudaSuccess)
     return bail(fail(BLAST_CF_ENOMEM, "workspace allocation"));
   for (auto &e : h->ev)
     if (cudaEventCreate(&e) != cudaSuccess) return bail(fail(BLAST_CF_ECUDA, "event create"));
-  if (getenv("BLAST_CF_PROFILE") && cudaMalloc(&h->d_prof, std::max(h->ncta, 1) * 16 * sizeof(long long)) != cudaSuccess)
+  if (getenv("BLAST_CF_PROFILE") && cudaMalloc(&h->d_prof, std::max<int64_t>(h->ncta_cap, 1) * 16 * sizeof(long long)) != cudaSuccess)
     return bail(fail(BLAST_CF_ENOMEM, "profile buffer"));
   *out = h;
   return BLAST_CF_OK;
@@ -704,6 +710,46 @@ int blast_cf_eval_loopback(blast_cf *const *hs, int n, const double *const *x, c
     CUDA_TRY(cudaStreamSynchronize(hs[r]->stream));
   }
   return check_async(hs[0]);
+}
+
+int blast_cf_autotune(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                      double *out_Fdot1, double *out_FTv, double *out_dt_min, int reps, double *ms_out, int capacity,
+                      int *num_candidates) {
+  if (!h || !num_candidates) return fail(BLAST_CF_EINVAL, "NULL argument");
+  const std::vector<KB1Variant> c = kb1_candidates(h->dim, h->k);
+  *num_candidates = (int)c.size();
+  if (reps < 1) reps = 3;
+  cudaEvent_t e0, e1;
+  CUDA_TRY(cudaEventCreate(&e0));
+  CUDA_TRY(cudaEventCreate(&e1));
+  int best = 0;
+  float best_ms = 1e30f;
+  int rc = BLAST_CF_OK;
+  for (size_t i = 0; i < c.size() && !rc; ++i) {
+    if ((rc = apply_variant(h, c[i]))) break;
+    if ((rc = blast_cf_eval(h, x, v, e, rho0detJ0, out_Fdot1, out_FTv, out_dt_min))) break;   // warm-up
+    cudaEventRecord(e0, h->stream);
+    for (int r = 0; r < reps && !rc; ++r) rc = blast_cf_eval(h, x, v, e, rho0detJ0, out_Fdot1, out_FTv, out_dt_min);
+    cudaEventRecord(e1, h->stream);
+    if (cudaEventSynchronize(e1) != cudaSuccess) { rc = fail(BLAST_CF_ECUDA, "autotune timing"); break; }
+    float ms = 0.0f;
+    cudaEventElapsedTime(&ms, e0, e1);
+    ms /= reps;
+    if (ms_out && (int)i < capacity) ms_out[i] = ms;
+    if (ms < best_ms) { best_ms = ms; best = (int)i; }
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  if (rc) return rc;
+  return c.empty() ? BLAST_CF_OK : apply_variant(h, c[best]);
+}
+
+const char *blast_cf_variant_name(const blast_cf *h, int index) {
+  if (!h) return "";
+  if (index < 0) return h->var.name ? h->var.name : "";
+  static thread_local std::vector<KB1Variant> c;
+  c = kb1_candidates(h->dim, h->k);
+  return index < (int)c.size() ? c[index].name : "";
 }
 
 int blast_cf_get_info(const blast_cf *h, blast_cf_info *info) {

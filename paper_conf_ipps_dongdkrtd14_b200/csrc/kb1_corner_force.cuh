@@ -59,7 +59,11 @@ struct Dims3 {
   static constexpr int SZ_U_FWD = 3 * NF * N * P + N * T;          // U, UE
   static constexpr int SZ_U_BCK = 2 * D * P * P + T * T;           // ZB/ZG, ZE
   static constexpr int SZ_U = SZ_U_FWD > SZ_U_BCK ? SZ_U_FWD : SZ_U_BCK;
-  static constexpr int ZONE = SZ_X + SZ_E + SZ_ACCF + SZ_ACCE + SZ_J0 + SZ_S + SZ_P + SZ_T + SZ_U;
+  // two reused regions per zone:  A = T/TE -> S/Pq -> Z/ZE,  B = U/UE -> Y/YE
+  static constexpr int SZ_A0 = SZ_T_FWD > SZ_S + SZ_P ? SZ_T_FWD : SZ_S + SZ_P;
+  static constexpr int SZ_A = SZ_A0 > SZ_U_BCK ? SZ_A0 : SZ_U_BCK;
+  static constexpr int SZ_B = SZ_U_FWD > SZ_T_BCK ? SZ_U_FWD : SZ_T_BCK;
+  static constexpr int ZONE = SZ_X + SZ_E + SZ_ACCF + SZ_ACCE + SZ_J0 + SZ_A + SZ_B;
   static constexpr int TAB = 2 * N * P + N * T + N;
 };
 
@@ -85,11 +89,9 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
   double *sAF = sE + ZPC * Dm::SZ_E;              // [ZPC][3][NK]
   double *sAE = sAF + ZPC * Dm::SZ_ACCF;          // [ZPC][NT]
   double *sJ0 = sAE + ZPC * Dm::SZ_ACCE;          // [ZPC][9]
-  double *sS = sJ0 + ZPC * Dm::SZ_J0;             // [ZPC][9][NS]
-  double *sP = sS + ZPC * Dm::SZ_S;               // [ZPC][NS]
-  double *sTr = sP + ZPC * Dm::SZ_P;              // [ZPC][SZ_T]  TB/TG/TE  | Y/YE
-  double *sUr = sTr + ZPC * Dm::SZ_T;             // [ZPC][SZ_U]  U/UE      | ZB/ZG/ZE
-  double *sRed = sUr + ZPC * Dm::SZ_U;            // [32]
+  double *sRA = sJ0 + ZPC * Dm::SZ_J0;             // [ZPC][SZ_A]  TB/TG/TE | S[9][NS] Pq[NS] | ZB/ZG/ZE
+  double *sRB = sRA + ZPC * Dm::SZ_A;               // [ZPC][SZ_B]  U/UE     | Y/YE
+  double *sRed = sRB + ZPC * Dm::SZ_B;             // [32]
 
   const int tid = threadIdx.x;
   const int64_t zone0 = (int64_t)blockIdx.x * ZPC;
@@ -150,7 +152,7 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
         tb = fma(sB[q2 * P + a2], xv, tb);
         tg = fma(sG[q2 * P + a2], xv, tg);
       }
-      double *Tz = sTr + zl * Dm::SZ_T;
+      double *Tz = sRA + zl * Dm::SZ_A;
       Tz[f * P2 + r] = tb;
       Tz[NF * P2 + f * P2 + r] = tg;
     }
@@ -160,7 +162,7 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
       double te = 0.0;
 #pragma unroll
       for (int j2 = 0; j2 < T; ++j2) te = fma(sPhi[q2 * T + j2], Ez[j2 * T2], te);
-      sTr[zl * Dm::SZ_T + 2 * NF * P2 + r] = te;
+      sRA[zl * Dm::SZ_A + 2 * NF * P2 + r] = te;
     }
     __syncthreads();
     // ---- stage B: contract a1 -> q1 --------------------------------------------------------------
@@ -168,7 +170,7 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
       const int zl = i / (NF * N * P), rr = i - zl * (NF * N * P);
       const int f = rr / (N * P), r2 = rr - f * (N * P);
       const int qq1 = r2 / P, a0 = r2 - qq1 * P;
-      const double *Tz = sTr + zl * Dm::SZ_T;
+      const double *Tz = sRA + zl * Dm::SZ_A;
       const double *TB = Tz + f * P2 + a0, *TG = Tz + NF * P2 + f * P2 + a0;
       double u0 = 0.0, u1 = 0.0, u2 = 0.0;
 #pragma unroll
@@ -179,7 +181,7 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
         u1 = fma(g, tb, u1);
         u2 = fma(b, tg, u2);
       }
-      double *Uz = sUr + zl * Dm::SZ_U + f * 3 * N * P;
+      double *Uz = sRB + zl * Dm::SZ_B + f * 3 * N * P;
       Uz[0 * N * P + r2] = u0;
       Uz[1 * N * P + r2] = u1;
       Uz[2 * N * P + r2] = u2;
@@ -187,16 +189,16 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
     for (int i = tid; i < ZPC * N * T; i += NTH) {
       const int zl = i / (N * T), r = i - zl * (N * T);
       const int qq1 = r / T, j0 = r - qq1 * T;
-      const double *TE = sTr + zl * Dm::SZ_T + 2 * NF * P2 + j0;
+      const double *TE = sRA + zl * Dm::SZ_A + 2 * NF * P2 + j0;
       double ue = 0.0;
 #pragma unroll
       for (int j1 = 0; j1 < T; ++j1) ue = fma(sPhi[qq1 * T + j1], TE[j1 * T], ue);
-      sUr[zl * Dm::SZ_U + 3 * NF * N * P + r] = ue;
+      sRB[zl * Dm::SZ_B + 3 * NF * N * P + r] = ue;
     }
     __syncthreads();
     // ---- stage C + point evaluation --------------------------------------------------------------
     if (has_point) {
-      const double *Uz = sUr + my_zl * Dm::SZ_U;
+      const double *Uz = sRB + my_zl * Dm::SZ_B;
       double Jm[3][3], Gv[3][3];
 #pragma unroll
       for (int f = 0; f < NF; ++f) {
@@ -221,12 +223,12 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
       const double alpha = sW[q0] * sW[q1] * sW[q2];
       PointOut<3> o;
       point_eval3(Jm, Gv, eq, R, alpha, gamma, sJ0 + my_zl * 9, a.ph, o);
-      double *S = sS + my_zl * Dm::SZ_S + my_qq;
+      double *S = sRA + my_zl * Dm::SZ_A + my_qq;
 #pragma unroll
       for (int c = 0; c < 3; ++c)
 #pragma unroll
         for (int d = 0; d < 3; ++d) S[(c * 3 + d) * NS] = o.S[c][d];
-      sP[my_zl * NS + my_qq] = o.P;
+      sRA[my_zl * Dm::SZ_A + Dm::SZ_S + my_qq] = o.P;
       if (a.Sq != nullptr && active) {
 #pragma unroll
         for (int c = 0; c < 9; ++c) a.Sq[(my_z * Dm::NQ + q) * 9 + c] = o.S[c / 3][c % 3];
@@ -242,7 +244,7 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
       const int zl = i / (3 * N * P), rr = i - zl * (3 * N * P);
       const int c = rr / (N * P), r2 = rr - c * (N * P);
       const int qq1 = r2 / P, a0 = r2 - qq1 * P;
-      const double *S = sS + zl * Dm::SZ_S + qq1 * N;
+      const double *S = sRA + zl * Dm::SZ_A + qq1 * N;
       double y0 = 0.0, y1 = 0.0, y2 = 0.0;
 #pragma unroll
       for (int qq0 = 0; qq0 < N; ++qq0) {
@@ -251,7 +253,7 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
         y1 = fma(b, S[(c * 3 + 1) * NS + qq0], y1);
         y2 = fma(b, S[(c * 3 + 2) * NS + qq0], y2);
       }
-      double *Y = sTr + zl * Dm::SZ_T + c * 3 * N * P;
+      double *Y = sRB + zl * Dm::SZ_B + c * 3 * N * P;
       Y[0 * N * P + r2] = y0;
       Y[1 * N * P + r2] = y1;
       Y[2 * N * P + r2] = y2;
@@ -259,11 +261,11 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
     for (int i = tid; i < ZPC * N * T; i += NTH) {
       const int zl = i / (N * T), r = i - zl * (N * T);
       const int qq1 = r / T, j0 = r - qq1 * T;
-      const double *Pz = sP + zl * NS + qq1 * N;
+      const double *Pz = sRA + zl * Dm::SZ_A + Dm::SZ_S + qq1 * N;
       double ye = 0.0;
 #pragma unroll
       for (int qq0 = 0; qq0 < N; ++qq0) ye = fma(sPhi[qq0 * T + j0], Pz[qq0], ye);
-      sTr[zl * Dm::SZ_T + 9 * N * P + r] = ye;
+      sRB[zl * Dm::SZ_B + 9 * N * P + r] = ye;
     }
     __syncthreads();
     // ---- stage B^T: contract q1 -> a1 -------------------------------------------------------------
@@ -271,7 +273,7 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
       const int zl = i / (3 * P2), rr = i - zl * (3 * P2);
       const int c = rr / P2, r = rr - c * P2;
       const int a1 = r / P, a0 = r - a1 * P;
-      const double *Y = sTr + zl * Dm::SZ_T + c * 3 * N * P + a0;
+      const double *Y = sRB + zl * Dm::SZ_B + c * 3 * N * P + a0;
       double zbv = 0.0, zgv = 0.0;
 #pragma unroll
       for (int qq1 = 0; qq1 < N; ++qq1) {
@@ -280,18 +282,18 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
         zbv = fma(g, Y[N * P + qq1 * P], zbv);
         zgv = fma(b, Y[2 * N * P + qq1 * P], zgv);
       }
-      double *Zr = sUr + zl * Dm::SZ_U;
+      double *Zr = sRA + zl * Dm::SZ_A;
       Zr[c * P2 + r] = zbv;
       Zr[3 * P2 + c * P2 + r] = zgv;
     }
     for (int i = tid; i < ZPC * T2; i += NTH) {
       const int zl = i / T2, r = i - zl * T2;
       const int j1 = r / T, j0 = r - j1 * T;
-      const double *YE = sTr + zl * Dm::SZ_T + 9 * N * P + j0;
+      const double *YE = sRB + zl * Dm::SZ_B + 9 * N * P + j0;
       double ze = 0.0;
 #pragma unroll
       for (int qq1 = 0; qq1 < N; ++qq1) ze = fma(sPhi[qq1 * T + j1], YE[qq1 * T], ze);
-      sUr[zl * Dm::SZ_U + 6 * P2 + r] = ze;
+      sRA[zl * Dm::SZ_A + 6 * P2 + r] = ze;
     }
     __syncthreads();
     // ---- stage A^T: accumulate q2 -> a2 -----------------------------------------------------------
@@ -299,16 +301,15 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
       const int zl = i / (3 * NK), rr = i - zl * (3 * NK);
       const int c = rr / NK, r3 = rr - c * NK;
       const int a2 = r3 / P2, r = r3 - a2 * P2;
-      const double *Zr = sUr + zl * Dm::SZ_U;
+      const double *Zr = sRA + zl * Dm::SZ_A;
       sAF[i] = fma(sB[q2 * P + a2], Zr[c * P2 + r], fma(sG[q2 * P + a2], Zr[3 * P2 + c * P2 + r], sAF[i]));
     }
     for (int i = tid; i < ZPC * NT; i += NTH) {
       const int zl = i / NT, r3 = i - zl * NT;
       const int j2 = r3 / T2, r = r3 - j2 * T2;
-      sAE[i] = fma(sPhi[q2 * T + j2], sUr[zl * Dm::SZ_U + 6 * P2 + r], sAE[i]);
+      sAE[i] = fma(sPhi[q2 * T + j2], sRA[zl * Dm::SZ_A + 6 * P2 + r], sAE[i]);
     }
-    // no barrier needed here: the next stage A writes only the T region (read last in stage B^T,
-    // before the previous barrier); the U region read above is next written in stage B, after a barrier
+    __syncthreads();   // region A (Z read above) is overwritten by the next slab's stage A
   }
   __syncthreads();
   // ---- outputs ----------------------------------------------------------------------------------

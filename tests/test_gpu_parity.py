@@ -219,3 +219,31 @@ def test_multi_material_gamma(orc):
     m, s = synth.config("C5", "S1", N=(6, 3, 3), k=2)
     assert len(np.unique(m.zone_mat)) == 3
     check(m, s, orc)
+
+
+CANDIDATES = {2: ["v2.z4", "v3.z4", "v1.z16"], 3: ["v3.z2", "v2.z2", "v1.z8"],
+              4: ["v4.m0", "v4.m1", "v3.z1", "v2.z1", "v1.z4"]}
+
+
+@pytest.mark.parametrize("k,name", [(k, n) for k, ns in CANDIDATES.items() for n in ns])
+def test_every_kernel_variant(orc, k, name, monkeypatch):
+    """Every candidate corner-force kernel (BLAST_CF_KB1 picks it at create) meets the parity bar."""
+    monkeypatch.setenv("BLAST_CF_KB1", name)
+    m, s = synth.config("C4", "S1", N=(5, 3, 2), k=k)
+    h, _, _ = check(m, s, orc)
+    assert h.variant == name
+
+
+def test_autotune_picks_a_candidate_and_keeps_parity(orc):
+    torch = _torch()
+    m, s = synth.config("C4", "S1", N=(6, 5, 4))
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    h = cf.from_synth(m)
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    x, v, e, r = t(s.x), t(s.v), t(s.e), t(s.rho0detJ0)
+    ms = h.autotune(x, v, e, r, reps=2)
+    assert set(ms) == set(CANDIDATES[4]) and all(val > 0 for val in ms.values())
+    assert h.variant == min(ms, key=ms.get)
+    F1, FTv, dt = (o.cpu().numpy() for o in h.eval(x, v, e, r))
+    ro = orc.evaluate(m, s)
+    assert rel(F1, ro.F1) <= TOL and rel(FTv, ro.FTv) <= TOL and abs(float(dt[0]) - ro.dt_min) <= TOL * ro.dt_min
