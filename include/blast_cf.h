@@ -182,6 +182,79 @@ int blast_cf_exchange_plan(int32_t rank, int32_t num_neighbors, const int32_t *n
 int blast_cf_nccl_unique_id_size(void);
 int blast_cf_nccl_get_unique_id(void *out);
 
+/* ---------------------------------------------------------------------------------------------
+ * Time integrator around the corner force.
+ *
+ * The semi-discrete system (eqs (1)-(3))
+ *     M_V dv/dt = -F.1,      M_E de/dt = F^T v,      dx/dt = v
+ * with the kinematic mass matrix (M_V)_ab = int rho W_a W_b (global, sparse, solved by CG each step:
+ * PAPER.md:193-198 and kernel 9 "CUDA-PCG", 405-413) and the thermodynamic mass matrix
+ * (M_E)_ij = int rho phi_i phi_j (block diagonal, inverse precomputed once: PAPER.md:198-205, kernel 11,
+ * 414-420).  rho|J| = rho0|J0| makes both time-independent.  Design:
+ *   - M_V is never assembled: its action is evaluated matrix-free per zone by sum factorization
+ *     (B^T diag(alpha rho0|J0|) B) and gathered to the nodes in ascending zone id — deterministic;
+ *     Jacobi-preconditioned CG with device-resident scalars, dim systems in lockstep;
+ *   - M_E^{-1}: zones whose rho0|J0| is constant over the zone use the tensor-product inverse
+ *     (M1^{-1} (x) M1^{-1} (x) M1^{-1}) / (rho0|J0|) (sum-factorized); other zones a dense per-zone
+ *     inverse computed at create in long double;
+ *   - F^T Vbar is applied from the S(q) the corner-force kernel stores (no F_z is ever formed);
+ *   - time stepping: the RK2-average scheme (reading R22), which conserves the discrete total
+ *     energy 1/2 v^T M_V v + sum_z 1^T M_E e_z up to the CG tolerance (the paper's Table 6 check,
+ *     PAPER.md:894-900); reflecting walls v.n = 0 on the bounding box of x0 (reading R23).
+ * Single GPU (mesh->nranks == 1) in this version.
+ * --------------------------------------------------------------------------------------------- */
+typedef struct blast_cf_rk2 blast_cf_rk2; /* opaque; borrows the corner-force handle h (same stream) */
+
+typedef struct {
+  double cg_rel_tol;      /* 1e-14: per component, stop when ||r|| <= tol * ||b|| (residual 2-norm) */
+  int32_t cg_max_iter;    /* 500 */
+  int32_t cg_check_every; /* 8: iterations between host-side convergence checks */
+  int32_t wall_bc;        /* 1: v . n = 0 on the walls of the bounding box of x0; 0: free */
+} blast_cf_rk2_opts;
+
+void blast_cf_rk2_default_opts(blast_cf_rk2_opts *o);
+
+/* Create the integrator for handle h.  mesh: the mesh h was created from (HOST pointers; x0 gives the
+ * walls).  rho0detJ0: HOST [num_zones][Nq], copied (the integrator evaluates the force with this copy).
+ * Allocates all device workspace.  BLAST_CF_EUNSUPPORTED for nranks > 1, or for dense M_E^{-1} zones
+ * beyond 2^34 long-double flops at create. */
+int blast_cf_rk2_create(blast_cf *h, const blast_cf_mesh *mesh, const double *rho0detJ0,
+                        const blast_cf_rk2_opts *opts, blast_cf_rk2 **out);
+
+/* One RK2-average step of length dt, IN PLACE on the caller's DEVICE arrays x, v [dim][num_nodes] and
+ * e [num_zones][Nt]:
+ *   dv0 = -M_V^{-1} F(S0).1,  Vb = v0 + dt/2 dv0,  de0 = M_E^{-1} F(S0)^T Vb,
+ *   S_half = (x0 + dt/2 Vb, Vb, e0 + dt/2 de0),
+ *   dv1 = -M_V^{-1} F(S_half).1,  Vb = v0 + dt/2 dv1,  de1 = M_E^{-1} F(S_half)^T Vb,
+ *   x1 = x0 + dt Vb,  v1 = v0 + dt dv1,  e1 = e0 + dt de1.
+ * dt_est (HOST, may be NULL): min of the two evaluations' dt estimates (the caller's dt control);
+ * cg_iters (HOST, may be NULL): CG iterations of the two solves (max over components, summed).
+ * Synchronous (the CG convergence checks read device scalars). */
+int blast_cf_rk2_step(blast_cf_rk2 *s, double *x, double *v, double *e, double dt, double *dt_est,
+                      int32_t *cg_iters);
+
+/* March to t_final (at most max_steps accepted steps) with the step-size control of reading R24: a step
+ * whose dt estimate falls below the dt it used is undone and retried with 0.85 dt; an accepted step
+ * whose estimate is >= 1.25 dt grows dt by 2 %.  *dt (HOST, in/out): the first trial dt, on return the
+ * next one.  t_reached, steps, rejected (HOST, may be NULL).  x, v, e DEVICE, advanced in place. */
+int blast_cf_rk2_advance(blast_cf_rk2 *s, double *x, double *v, double *e, double t_final, int32_t max_steps,
+                         double *dt, double *t_reached, int32_t *steps, int32_t *rejected);
+
+/* The two rates of the system at state (x, v, e) (DEVICE arrays): out_dvdt = -M_V^{-1} F.1 (walls
+ * applied), out_dedt = M_E^{-1} F^T vbar (vbar NULL: v), out_dt = the evaluation's dt estimate (HOST).
+ * Synchronous.  The building block of blast_cf_rk2_step, exposed for tests. */
+int blast_cf_rk2_rates(blast_cf_rk2 *s, const double *x, const double *v, const double *e, const double *vbar,
+                       double *out_dvdt, double *out_dedt, double *out_dt, int32_t *cg_iters);
+
+/* Tests: out = M_V u per component ([dim][num_nodes], DEVICE; no wall mask). */
+int blast_cf_rk2_mass_apply(blast_cf_rk2 *s, const double *u, double *out);
+
+/* Discrete energies (HOST outputs): kinetic = 1/2 sum_c v_c^T M_V v_c, internal = sum_z 1^T M_E e_z.
+ * v, e DEVICE.  Deterministic.  Synchronous. */
+int blast_cf_rk2_energy(blast_cf_rk2 *s, const double *v, const double *e, double *kinetic, double *internal);
+
+int blast_cf_rk2_destroy(blast_cf_rk2 *s);
+
 #ifdef __cplusplus
 }
 #endif

@@ -152,3 +152,21 @@ class RK2Avg:
         Vb = v + 0.5 * dt * dv
         de = self.de_dt(r1, Vb)
         return x + dt * Vb, v + dt * dv, e + dt * de, min(r0.dt_min, r1.dt_min)
+
+    def advance(self, x, v, e, t_final, dt, max_steps):
+        """Step to t_final with the step-size control of reading R24 (Laghos's rule): a step whose
+        dt estimate (min over its two force evaluations) falls below the dt it used is rejected and
+        retried with 0.85 dt; an accepted step with estimate >= 1.25 dt grows dt by 2 %."""
+        t, steps, rejected = 0.0, 0, 0
+        while t < t_final and steps < max_steps:
+            dt_use = min(dt, t_final - t)
+            x1, v1, e1, dte = self.step(x, v, e, dt_use)
+            if dte < dt_use:
+                dt = 0.85 * dt_use
+                rejected += 1
+                continue
+            x, v, e = x1, v1, e1
+            t += dt_use
+            steps += 1
+            dt = 1.02 * dt_use if dte >= 1.25 * dt_use else dt_use
+        return x, v, e, t, dt, steps, rejected

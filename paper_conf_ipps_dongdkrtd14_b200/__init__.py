@@ -48,6 +48,11 @@ class Params(ctypes.Structure):
                 ("use_vorticity", ctypes.c_int32)]
 
 
+class RK2Opts(ctypes.Structure):
+    _fields_ = [("cg_rel_tol", ctypes.c_double), ("cg_max_iter", ctypes.c_int32), ("cg_check_every", ctypes.c_int32),
+                ("wall_bc", ctypes.c_int32)]
+
+
 class Info(ctypes.Structure):
     _fields_ = [("dim", ctypes.c_int32), ("order", ctypes.c_int32), ("nq", ctypes.c_int32), ("nk", ctypes.c_int32),
                 ("nt", ctypes.c_int32), ("num_zones", ctypes.c_int64), ("num_nodes", ctypes.c_int64),
@@ -98,7 +103,19 @@ def lib():
     L.blast_cf_autotune.argtypes = [vp] * 8 + [ctypes.c_int, vp, ctypes.c_int, ctypes.POINTER(ctypes.c_int)]
     L.blast_cf_variant_name.argtypes = [vp, ctypes.c_int]
     L.blast_cf_variant_name.restype = ctypes.c_char_p
-    for f in ("blast_cf_create", "blast_cf_eval", "blast_cf_eval_host", "blast_cf_eval_debug_Fz", "blast_cf_get_info",
+    L.blast_cf_rk2_default_opts.argtypes = [ctypes.POINTER(RK2Opts)]
+    L.blast_cf_rk2_create.argtypes = [vp, ctypes.POINTER(_Mesh), vp, ctypes.POINTER(RK2Opts), vp]
+    L.blast_cf_rk2_step.argtypes = [vp, vp, vp, vp, ctypes.c_double, ctypes.POINTER(ctypes.c_double),
+                                    ctypes.POINTER(i32)]
+    L.blast_cf_rk2_rates.argtypes = [vp] * 7 + [ctypes.POINTER(ctypes.c_double), ctypes.POINTER(i32)]
+    L.blast_cf_rk2_mass_apply.argtypes = [vp, vp, vp]
+    L.blast_cf_rk2_advance.argtypes = [vp, vp, vp, vp, ctypes.c_double, i32, ctypes.POINTER(ctypes.c_double),
+                                       ctypes.POINTER(ctypes.c_double), ctypes.POINTER(i32), ctypes.POINTER(i32)]
+    L.blast_cf_rk2_energy.argtypes = [vp, vp, vp, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]
+    L.blast_cf_rk2_destroy.argtypes = [vp]
+    for f in ("blast_cf_rk2_create", "blast_cf_rk2_step", "blast_cf_rk2_rates", "blast_cf_rk2_mass_apply",
+              "blast_cf_rk2_energy", "blast_cf_rk2_destroy", "blast_cf_rk2_advance",
+              "blast_cf_create", "blast_cf_eval", "blast_cf_eval_host", "blast_cf_eval_debug_Fz", "blast_cf_get_info",
               "blast_cf_set_timing", "blast_cf_kernel_times", "blast_cf_destroy", "blast_cf_nccl_unique_id_size",
               "blast_cf_nccl_get_unique_id", "blast_cf_exchange_plan", "blast_cf_debug_cta_dt",
               "blast_cf_debug_stage_clocks", "blast_cf_eval_loopback", "blast_cf_autotune"):
@@ -189,6 +206,7 @@ class CornerForce:
             _check(L.blast_cf_create(ctypes.byref(m), self.order, self.dim, ctypes.byref(self.params),
                                      ctypes.c_void_p(self.stream.cuda_stream), uid, ctypes.byref(h)), "blast_cf_create")
         self._h = h
+        self._mesh_struct = m   # the arrays it points to live in self (the integrator re-reads x0)
         self.info = self.get_info()
 
     # ------------------------------------------------------------------
@@ -302,6 +320,95 @@ class CornerForce:
     def close(self):
         if getattr(self, "_h", None):
             lib().blast_cf_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def rk2_default_opts() -> RK2Opts:
+    o = RK2Opts()
+    lib().blast_cf_rk2_default_opts(ctypes.byref(o))
+    return o
+
+
+class RK2:
+    """The time integrator around a CornerForce handle (blast_cf_rk2_*).
+
+    State arrays are torch.cuda float64 tensors x, v [dim][nodes], e [Z][Nt], advanced in place.
+    """
+
+    def __init__(self, cf: CornerForce, rho0detJ0: np.ndarray, opts: Optional[RK2Opts] = None, **kw):
+        self.cf = cf
+        self._R = np.ascontiguousarray(rho0detJ0, dtype=np.float64)
+        assert self._R.shape == (cf.num_zones, cf.nq)
+        self.opts = opts if opts is not None else rk2_default_opts()
+        for k_, v_ in kw.items():
+            setattr(self.opts, k_, v_)
+        h = ctypes.c_void_p()
+        _check(lib().blast_cf_rk2_create(cf._h, ctypes.byref(cf._mesh_struct), self._R.ctypes.data,
+                                         ctypes.byref(self.opts), ctypes.byref(h)), "blast_cf_rk2_create")
+        self._h = h
+
+    def _shapes(self):
+        c = self.cf
+        return (c.dim, c.num_nodes), (c.num_zones, c.nt)
+
+    def step(self, x, v, e, dt: float):
+        """One RK2-average step in place; returns (dt estimate, CG iterations)."""
+        sx, se = self._shapes()
+        d = ctypes.c_double(0.0)
+        it = ctypes.c_int32(0)
+        _check(lib().blast_cf_rk2_step(self._h, self.cf._dev(x, sx), self.cf._dev(v, sx), self.cf._dev(e, se),
+                                       float(dt), ctypes.byref(d), ctypes.byref(it)), "blast_cf_rk2_step")
+        return d.value, it.value
+
+    def advance(self, x, v, e, t_final: float, dt: float, max_steps: int):
+        """March in place to t_final (<= max_steps accepted steps) with the R24 step control.
+        Returns (t reached, next dt, steps, rejected)."""
+        sx, se = self._shapes()
+        d, tr = ctypes.c_double(dt), ctypes.c_double(0.0)
+        ns, nr = ctypes.c_int32(0), ctypes.c_int32(0)
+        _check(lib().blast_cf_rk2_advance(self._h, self.cf._dev(x, sx), self.cf._dev(v, sx), self.cf._dev(e, se),
+                                          float(t_final), int(max_steps), ctypes.byref(d), ctypes.byref(tr),
+                                          ctypes.byref(ns), ctypes.byref(nr)), "blast_cf_rk2_advance")
+        return tr.value, d.value, ns.value, nr.value
+
+    def rates(self, x, v, e, vbar=None):
+        """(dv/dt, de/dt, dt estimate, CG iterations) at state (x, v, e); de/dt uses vbar (default v)."""
+        import torch
+        sx, se = self._shapes()
+        dv = torch.empty(sx, dtype=torch.float64, device=self.cf.device)
+        de = torch.empty(se, dtype=torch.float64, device=self.cf.device)
+        d = ctypes.c_double(0.0)
+        it = ctypes.c_int32(0)
+        _check(lib().blast_cf_rk2_rates(self._h, self.cf._dev(x, sx), self.cf._dev(v, sx), self.cf._dev(e, se),
+                                        None if vbar is None else self.cf._dev(vbar, sx), self.cf._dev(dv, sx),
+                                        self.cf._dev(de, se), ctypes.byref(d), ctypes.byref(it)), "blast_cf_rk2_rates")
+        return dv, de, d.value, it.value
+
+    def mass_apply(self, u):
+        import torch
+        sx, _ = self._shapes()
+        out = torch.empty(sx, dtype=torch.float64, device=self.cf.device)
+        _check(lib().blast_cf_rk2_mass_apply(self._h, self.cf._dev(u, sx), self.cf._dev(out, sx)),
+               "blast_cf_rk2_mass_apply")
+        return out
+
+    def energy(self, v, e):
+        """(kinetic, internal) discrete energies."""
+        sx, se = self._shapes()
+        ke, ie = ctypes.c_double(0.0), ctypes.c_double(0.0)
+        _check(lib().blast_cf_rk2_energy(self._h, self.cf._dev(v, sx), self.cf._dev(e, se), ctypes.byref(ke),
+                                         ctypes.byref(ie)), "blast_cf_rk2_energy")
+        return ke.value, ie.value
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib().blast_cf_rk2_destroy(self._h)
             self._h = None
 
     def __del__(self):

@@ -7,7 +7,8 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libblastcf.so")
-SOURCES = [os.path.join(CSRC, "blast_cf.cu")]
+SOURCES = [os.path.join(CSRC, "blast_cf.cu"), os.path.join(CSRC, "integrator.cu")]
+OBJDIR = os.path.join(HERE, "build")
 DEPS = [os.path.join(CSRC, f) for f in os.listdir(CSRC)] + [os.path.join(ROOT, "include", "blast_cf.h")]
 
 
@@ -27,7 +28,7 @@ def nccl_lib():
 
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
-              "-Xcompiler", "-fPIC", "-shared", "-Xptxas", "-warn-spills"]
+              "-Xcompiler", "-fPIC", "-Xptxas", "-warn-spills"]
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
@@ -35,12 +36,23 @@ def build(force: bool = False, verbose: bool = False) -> str:
         t = os.path.getmtime(LIB)
         if all(os.path.getmtime(d) <= t for d in DEPS):
             return LIB
+    os.makedirs(OBJDIR, exist_ok=True)
+    inc = ["-I", os.path.join(ROOT, "include"), "-I", nccl_include()]
+    objs, procs = [], []
+    for src in SOURCES:   # one object per translation unit, compiled in parallel
+        obj = os.path.join(OBJDIR, os.path.basename(src) + f".{os.getpid()}.o")
+        cmd = ["nvcc", *NVCC_FLAGS, *inc, "-c", "-o", obj, src]
+        if verbose:
+            cmd.insert(1, "-Xptxas=-v")
+            print(" ".join(cmd))
+        objs.append(obj)
+        procs.append(subprocess.Popen(cmd))
+    if any(p.wait() != 0 for p in procs):
+        raise subprocess.CalledProcessError(1, "nvcc")
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = ["nvcc", *NVCC_FLAGS, "-I", os.path.join(ROOT, "include"), "-I", nccl_include(), "-o", tmp, *SOURCES, "-ldl"]
-    if verbose:
-        cmd.insert(1, "-Xptxas=-v")
-        print(" ".join(cmd))
-    subprocess.check_call(cmd)
+    subprocess.check_call(["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", tmp, *objs, "-ldl"])
+    for o in objs:
+        os.remove(o)
     os.replace(tmp, LIB)
     return LIB
 

@@ -23,6 +23,7 @@
 #include "kb2_gather.cuh"
 #include "tables.h"
 #include "exchange.cuh"
+#include "internal.h"
 
 namespace {
 
@@ -617,6 +618,30 @@ static int eval_impl(blast_cf *h, const double *x, const double *v, const double
   if (h->timing) cudaEventRecord(h->ev[3], h->stream);
   return check_async(h);
 }
+
+}  // extern "C"
+
+namespace blastcf {
+
+int handle_view(const blast_cf *h, HandleView *o) {
+  if (!h || !o) return fail(BLAST_CF_EINVAL, "NULL argument");
+  o->dim = h->dim; o->k = h->k; o->nk = h->nk; o->nt = h->nt; o->nq = h->nq;
+  o->Z = h->Z; o->nn = h->nn; o->stream = h->stream; o->device = h->device;
+  o->zone_nodes = h->d_zone_nodes; o->ptr = h->d_ptr; o->ent = h->d_ent; o->tab = h->d_tab;
+  o->multi_rank = h->xch != nullptr;
+  return BLAST_CF_OK;
+}
+
+int eval_with_S(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                double *out_Fdot1, double *out_FTv, double *out_dt_min, double *Sq) {
+  return eval_impl(h, x, v, e, rho0detJ0, out_Fdot1, out_FTv, out_dt_min, Sq);
+}
+
+int set_error(int code, const char *msg) { return fail(code, "%s", msg); }
+
+}  // namespace blastcf
+
+extern "C" {
 
 int blast_cf_eval(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
                   double *out_Fdot1, double *out_FTv, double *out_dt_min) {
