@@ -20,6 +20,8 @@
 #include "kb1_v2.cuh"
 #include "kb1_v3.cuh"
 #include "kb1_v4.cuh"
+#include "kb1_v5.cuh"
+#include "kb1_v6.cuh"
 #include "kb2_gather.cuh"
 #include "tables.h"
 #include "exchange.cuh"
@@ -109,6 +111,27 @@ KB1Variant variant3v4() {
   using C = KB1V4Cfg<K, MODE>;
   return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v4<K, MODE>, (const void *)&kb1_v4_3d<K, MODE>, true, nullptr};
 }
+template <int K, int DIAG, int MODE>
+void launch3v5(const KB1Args &a, int grid, cudaStream_t s) {
+  using C = KB1V5Cfg<K, MODE>;
+  kb1_v5_3d<K, DIAG, MODE><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+}
+template <int K, int DIAG = 0, int MODE = 0>
+KB1Variant variant3v5() {
+  using C = KB1V5Cfg<K, MODE>;
+  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v5<K, DIAG, MODE>, (const void *)&kb1_v5_3d<K, DIAG, MODE>,
+                    true, nullptr};
+}
+template <int K, int DIAG>
+void launch3v6(const KB1Args &a, int grid, cudaStream_t s) {
+  using C = KB1V5Cfg<K>;
+  kb1_v6_3d<K, DIAG><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+}
+template <int K, int DIAG = 0>
+KB1Variant variant3v6() {
+  using C = KB1V5Cfg<K>;
+  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v6<K, DIAG>, (const void *)&kb1_v6_3d<K, DIAG>, true, nullptr};
+}
 template <int K, int ZPC, int MINB>
 KB1Variant variant3() {
   using C = KB1Cfg3<K, ZPC>;
@@ -133,7 +156,7 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
       case 2: add(variant3v2<2, 4, 3>(), "v2.z4"); add(variant3v3<2, 4, 2>(), "v3.z4"); add(variant3<2, 16, 2>(), "v1.z16"); break;
       case 3: add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
       case 4:
-        add(variant3v4<4, 0>(), "v4.m0"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
+        add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
@@ -160,9 +183,22 @@ KB1Variant select_variant(int dim, int k) {
   const std::vector<KB1Variant> c = kb1_candidates(dim, k);
   if (c.empty()) return KB1Variant{0, 0, 0, nullptr, nullptr, false, nullptr};
   const char *force = getenv("BLAST_CF_KB1");   // experiments: pick a candidate by name
-  if (force)
+  if (force) {
     for (const KB1Variant &x : c)
       if (strcmp(x.name, force) == 0) return x;
+    // timing diagnostics (wrong results by design; never candidates of the autotuner)
+    if (dim == 3 && k == 4) {
+      KB1Variant d;
+      if (strcmp(force, "v5.d1") == 0) { d = variant3v5<4, 1>(); d.name = "v5.d1"; return d; }
+      if (strcmp(force, "v5.d2") == 0) { d = variant3v5<4, 2>(); d.name = "v5.d2"; return d; }
+      if (strcmp(force, "v6.d1") == 0) { d = variant3v6<4, 1>(); d.name = "v6.d1"; return d; }
+      if (strcmp(force, "v6.d2") == 0) { d = variant3v6<4, 2>(); d.name = "v6.d2"; return d; }
+      if (strcmp(force, "v5.r1") == 0) { d = variant3v5<4, 0, 1>(); d.name = "v5.r1"; return d; }
+      if (strcmp(force, "v5.r2") == 0) { d = variant3v5<4, 0, 2>(); d.name = "v5.r2"; return d; }
+      if (strcmp(force, "v5.r1d1") == 0) { d = variant3v5<4, 1, 1>(); d.name = "v5.r1d1"; return d; }
+      if (strcmp(force, "v5.r2d1") == 0) { d = variant3v5<4, 1, 2>(); d.name = "v5.r2d1"; return d; }
+    }
+  }
   return c[0];
 }
 
@@ -595,7 +631,7 @@ static int eval_impl(blast_cf *h, const double *x, const double *v, const double
   a.x = x; a.v = v; a.e = e; a.rho0detJ0 = rho0detJ0;
   a.zone_nodes = h->d_zone_nodes; a.J0inv = h->d_J0inv; a.zone_gamma = h->d_gamma; a.tab = h->d_tab;
   a.Fz1 = h->d_Fz1; a.FTv = out_FTv; a.cta_dt = h->d_ctadt; a.Sq = Sq; a.prof = h->d_prof;
-  a.num_zones = h->Z; a.num_nodes = h->nn;
+  a.num_zones = h->Z; a.num_nodes = h->nn; a.zero = 0;
   a.ph.cfl = h->params.cfl; a.ph.q_quad = h->params.q_quad; a.ph.q_lin = h->params.q_lin;
   a.ph.eps_sw = h->params.eps_switch; a.ph.inv_2eps = 0.5 / h->params.eps_switch; a.ph.h0 = h->h0; a.ph.k = (double)h->k;
   a.ph.use_visc = h->params.use_viscosity; a.ph.use_vort = h->params.use_vorticity;

@@ -28,6 +28,7 @@ struct KB1Args {
   long long *prof;         // debug only: per-CTA clock64 stamps at the stage barriers [grid][16], else nullptr
   int64_t num_zones, num_nodes;
   CFPhys ph;
+  int32_t zero;            // always 0 (an offset the compiler cannot fold: kb1_v6.cuh)
 };
 
 __device__ __forceinline__ double block_min(double v, double *red) {
