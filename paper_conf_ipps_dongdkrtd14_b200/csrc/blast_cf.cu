@@ -156,7 +156,7 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
       case 2: add(variant3v2<2, 4, 3>(), "v2.z4"); add(variant3v3<2, 4, 2>(), "v3.z4"); add(variant3<2, 16, 2>(), "v1.z16"); break;
       case 3: add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
       case 4:
-        add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
+        add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
@@ -193,7 +193,6 @@ KB1Variant select_variant(int dim, int k) {
       if (strcmp(force, "v5.d2") == 0) { d = variant3v5<4, 2>(); d.name = "v5.d2"; return d; }
       if (strcmp(force, "v6.d1") == 0) { d = variant3v6<4, 1>(); d.name = "v6.d1"; return d; }
       if (strcmp(force, "v6.d2") == 0) { d = variant3v6<4, 2>(); d.name = "v6.d2"; return d; }
-      if (strcmp(force, "v5.r1") == 0) { d = variant3v5<4, 0, 1>(); d.name = "v5.r1"; return d; }
       if (strcmp(force, "v5.r2") == 0) { d = variant3v5<4, 0, 2>(); d.name = "v5.r2"; return d; }
       if (strcmp(force, "v5.r1d1") == 0) { d = variant3v5<4, 1, 1>(); d.name = "v5.r1d1"; return d; }
       if (strcmp(force, "v5.r2d1") == 0) { d = variant3v5<4, 1, 2>(); d.name = "v5.r2d1"; return d; }

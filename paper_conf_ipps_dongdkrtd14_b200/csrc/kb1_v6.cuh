@@ -79,6 +79,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K>::NTH, 1) kb1_v6_3d(const KB1Args a
   };
 
   for (int i = tid; i < 2 * N * P + N * T + N; i += Cfg::NTH) sTab[i] = __ldg(a.tab + i);
+  if (tid == 0) sRed[8] = 0.0;   // dt filter: best exact inverse dt of this CTA (point_eval3<true>)
 
   // ---------------- KW ----------------
   // node ids travel by cp.async into shared memory one zone ahead (a register copy of an __ldg result
@@ -415,8 +416,16 @@ __global__ void __launch_bounds__(KB1V5Cfg<K>::NTH, 1) kb1_v6_3d(const KB1Args a
       }
     const double w12 = sW[q1] * sW[q2];
     PointOut<3> oa, ob;
-    point_eval3(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa);
-    point_eval3(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob);
+    const double best = sRed[8];   // largest exact inverse dt found so far by this CTA (dt filter)
+    point_eval3<true>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best);
+    point_eval3<true>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best);
+    {
+      double mi = fmax(oa.inv, ob.inv);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) mi = fmax(mi, __shfl_xor_sync(0xffffffffu, mi, o));
+      if ((threadIdx.x & 31) == 0 && mi > best)
+        atomicMax(reinterpret_cast<unsigned long long *>(sRed + 8), (unsigned long long)__double_as_longlong(mi));
+    }
 #pragma unroll
     for (int cd = 0; cd < 9; ++cd) {     // in place over J: only this thread touches slots sa, sbi
       jb[cd * N3 + sa] = oa.S[cd / 3][cd % 3];
