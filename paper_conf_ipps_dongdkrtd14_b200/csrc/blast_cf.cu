@@ -22,6 +22,7 @@
 #include "kb1_v4.cuh"
 #include "kb1_v5.cuh"
 #include "kb1_v6.cuh"
+#include "kb1_v8.cuh"
 #include "kb2_gather.cuh"
 #include "tables.h"
 #include "exchange.cuh"
@@ -132,6 +133,16 @@ KB1Variant variant3v6() {
   using C = KB1V5Cfg<K>;
   return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v6<K, DIAG>, (const void *)&kb1_v6_3d<K, DIAG>, true, nullptr};
 }
+template <int K, int MINB>
+void launch3v8(const KB1Args &a, int grid, cudaStream_t s) {
+  using C = KB1V8Cfg<K>;
+  kb1_v8_3d<K, MINB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+}
+template <int K, int MINB>
+KB1Variant variant3v8() {
+  using C = KB1V8Cfg<K>;
+  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v8<K, MINB>, (const void *)&kb1_v8_3d<K, MINB>, false, nullptr};
+}
 template <int K, int ZPC, int MINB>
 KB1Variant variant3() {
   using C = KB1Cfg3<K, ZPC>;
@@ -161,8 +172,8 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
         break;
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
       case 6: add(variant3<6, 1, 2>(), "v1.z1m2"); add(variant3<6, 2, 1>(), "v1.z2"); break;
-      case 7: add(variant3<7, 1, 2>(), "v1.z1"); break;
-      case 8: add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
+      case 7: add(variant3v8<7, 1>(), "v8"); add(variant3<7, 1, 2>(), "v1.z1"); break;
+      case 8: add(variant3v8<8, 2>(), "v8"); add(variant3v8<8, 1>(), "v8.m1"); add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
     }
   } else {
     switch (k) {

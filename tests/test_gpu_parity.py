@@ -222,7 +222,8 @@ def test_multi_material_gamma(orc):
 
 
 CANDIDATES = {2: ["v2.z4", "v3.z4", "v1.z16"], 3: ["v3.z2", "v2.z2", "v1.z8"],
-              4: ["v4.m0", "v5.r1", "v5", "v6", "v4.m1", "v3.z1", "v2.z1", "v1.z4"]}
+              4: ["v5.r1", "v4.m0", "v5", "v6", "v4.m1", "v3.z1", "v2.z1", "v1.z4"],
+              7: ["v8", "v1.z1"], 8: ["v8", "v8.m1", "v1.z1m2", "v1.z1"]}
 
 
 @pytest.mark.parametrize("k,name", [(k, n) for k, ns in CANDIDATES.items() for n in ns])
