@@ -33,6 +33,9 @@ METRIC = "corner-force zones/s & FP64 GFLOP/s (Q4-Q3 3D Sedov) at 1/2/4/8 B200"
 FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12
 
 
+RK2_CONFIGS = ("C2",)   # configs whose step is the two-stage RK2 right-hand side
+
+
 def env_rank():
     return int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("LOCAL_RANK", "0"))
 
@@ -121,14 +124,17 @@ def workload_desc(name):
     return c["desc"]
 
 
-def load_traffic():
-    """dram bytes per KB1 launch from the committed ncu --set full summary (or None)."""
+def load_traffic(config, variant):
+    """dram bytes per KB1 launch from the committed ncu --set full summary of THIS config and KB1 variant
+    (profiles/kb1_ncu_summary.json, keyed by config); None when no capture of that kernel exists."""
     p = os.path.join(ROOT, "profiles", "kb1_ncu_summary.json")
     try:
-        d = json.load(open(p))
-        return d.get("dram_bytes_per_launch"), d.get("source")
+        d = json.load(open(p)).get(config)
     except Exception:
         return None, None
+    if not d or d.get("variant") != variant:
+        return None, None
+    return d.get("dram_bytes_per_launch"), d.get("source")
 
 
 def oracle_sample(mesh, st, seconds=15.0, max_zones=None):
@@ -212,9 +218,21 @@ def run_ours(args):
         h = cf.from_synth(mesh, part=part, nccl_uid=uid, stream=stream) if world > 1 else cf.from_synth(lmesh, stream=stream)
     info = h.info
     t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(dev)
-    x, v, e, r = t(lst.x), t(lst.v), t(lst.e), t(lst.rho0detJ0)
+    # the states one step evaluates: C2's step is the "full RK2 step RHS" = the corner force at the two
+    # RK2 stage states S1, S1b (R21); every other config's step is one evaluation
+    states = [lst]
+    if args.config in RK2_CONFIGS and args.state == "S1":
+        s1b = synth.config(args.config, "S1b")[1]
+        states.append(part.local_state(s1b) if world > 1 else s1b)
+    dev_states = [(t(s.x), t(s.v), t(s.e), t(s.rho0detJ0)) for s in states]
+    x, v, e, r = dev_states[0]
     out = h.alloc_outputs()
-    in_bytes = sum(a.numel() * 8 for a in (x, v, e, r))
+    in_bytes = sum(a.numel() * 8 for ds in dev_states for a in ds)
+    nev = len(dev_states)
+
+    def step():
+        for ds in dev_states:
+            h.eval(*ds, out=out)
 
     def barrier():
         torch.cuda.synchronize()
@@ -228,7 +246,7 @@ def run_ours(args):
         t_w = time.perf_counter()
         while True:   # W warm-up steps, then keep the GPU loaded until the sampler is up (>= 0.4 s)
             for _ in range(args.warmup):
-                h.eval(x, v, e, r, out=out)
+                step()
             torch.cuda.synchronize()
             if time.perf_counter() - t_w > 0.4:
                 break
@@ -237,7 +255,7 @@ def run_ours(args):
         e_start = meter.read_mj()
         ev0.record(stream)
         for _ in range(args.steps):
-            h.eval(x, v, e, r, out=out)
+            step()
         ev1.record(stream)
         barrier()
         e_end = meter.read_mj()
@@ -247,7 +265,7 @@ def run_ours(args):
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         ms = float(tt.item())
     ms_step = ms / args.steps
-    value = Zg * args.steps / (ms / 1e3)
+    value = Zg * nev * args.steps / (ms / 1e3)   # zone evaluations per second
 
     # per-kernel breakdown (separate pass, events on the library's stream)
     h.set_timing(True)
@@ -262,23 +280,26 @@ def run_ours(args):
     Zl = lmesh.num_zones
     flops_eval_local = info["flops_per_zone"] * Zl
     achieved_tf = flops_eval_local / (kb1_ms / 1e3) / 1e12
-    gflops_total = info["flops_per_zone"] * Zg / (ms_step / 1e3) / 1e9
-    traffic, tsrc = load_traffic()
+    gflops_total = info["flops_per_zone"] * Zg * nev / (ms_step / 1e3) / 1e9
+    traffic, tsrc = load_traffic(args.config, h.variant)
 
     # e2e through the public API with host buffers (pinned), H2D + eval + D2H inside the timed region
     e2e = None
     if not args.no_e2e:
-        hx = [torch.from_numpy(np.ascontiguousarray(a)).pin_memory() for a in (lst.x, lst.v, lst.e, lst.rho0detJ0)]
+        hxs = [[torch.from_numpy(np.ascontiguousarray(a)).pin_memory() for a in (s.x, s.v, s.e, s.rho0detJ0)]
+               for s in states]
         ho = (torch.empty(tuple(out[0].shape), dtype=torch.float64).pin_memory(),
               torch.empty(tuple(out[1].shape), dtype=torch.float64).pin_memory(),
               torch.empty(1, dtype=torch.float64).pin_memory())
-        h.eval_host(*hx, out=ho)
+        for hx in hxs:
+            h.eval_host(*hx, out=ho)
         barrier()
         k2 = max(3, min(args.steps, 10))
         a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a0.record(stream)
         for _ in range(k2):
-            h.eval_host(*hx, out=ho)
+            for hx in hxs:
+                h.eval_host(*hx, out=ho)
         a1.record(stream)
         barrier()
         ems = a0.elapsed_time(a1)
@@ -286,15 +307,15 @@ def run_ours(args):
             tt = torch.tensor([ems], device=dev, dtype=torch.float64)
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             ems = float(tt.item())
-        out_bytes = sum(o.numel() * 8 for o in ho)
-        e2e = {"value": Zg * k2 / (ems / 1e3), "unit": "zones/s", "h2d_bytes_per_step": int(in_bytes),
+        out_bytes = nev * sum(o.numel() * 8 for o in ho)
+        e2e = {"value": Zg * nev * k2 / (ems / 1e3), "unit": "zones/s", "h2d_bytes_per_step": int(in_bytes),
                "d2h_bytes_per_step": int(out_bytes), "ms_per_step": ems / k2}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         nz, tc, nthr = oracle_sample(mesh, st, seconds=args.cpu_seconds)
         cpu = {"value": nz / tc, "unit": "zones/s", "cores": nthr, "kind": "oracle",
-               "sample": f"first {nz} of {Zg} zones of the same C4 S1 state, one evaluation (plain C oracle, "
+               "sample": f"first {nz} of {Zg} zones of the same {args.config} {args.state} state, one evaluation (plain C oracle, "
                          f"OpenMP over zones, serial assembly), {tc:.1f} s"}
 
     energy = None
@@ -308,21 +329,22 @@ def run_ours(args):
             "metric": METRIC, "value": value, "unit": "zones/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"{args.config}: {workload_desc(args.config)}", "state": args.state,
-                       "zones": Zg, "order": mesh.order, "dim": mesh.dim,
+            "config": {"workload": f"{args.config}: {workload_desc(args.config)}",
+                       "state": "+".join(["S1", "S1b"][:nev]) if nev > 1 else args.state,
+                       "evals_per_step": nev, "zones": Zg, "order": mesh.order, "dim": mesh.dim,
                        "parallelism": f"domain decomposition {synth.block_dims(mesh.dim, world)}" if world > 1 else "single GPU",
                        "l2": f"inputs larger than L2 ({in_bytes / 1e6:.0f} MB of inputs per rank + "
                              f"{Zl * info['nk'] * mesh.dim * 8 / 1e6:.0f} MB zone-local buffer vs 126 MB L2); no flush"},
             "gflops": gflops_total,
             "roofline": {"bound": "alu", "achieved": achieved_tf, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
                          "frac": achieved_tf / FP64_PEAK_TFLOPS, "traffic": traffic,
-                         "kernel": "KB1 (fused corner force)",
+                         "kernel": f"KB1 (fused corner force, variant {h.variant})",
                          "kernel_ms": kb1_ms, "kb2_ms": float(kb[1]), "exchange_ms": float(kb[2]),
                          "flops_per_zone": info["flops_per_zone"],
                          "peak_note": "FP64 ALU: 148 SM x 64 FMA/clk x 2 x 1.965 GHz (measured DFMA 34.2 / DMMA 37.1 TF)",
                          "traffic_source": tsrc},
             "e2e": e2e,
-            "gpu_launches": int(info["kernels_per_eval"] * args.steps),
+            "gpu_launches": int(info["kernels_per_eval"] * nev * args.steps),
             "energy": energy,
             "clocks": clocks,
             "cpu_baseline": cpu,
