@@ -22,6 +22,7 @@
 #include "kb1_v4.cuh"
 #include "kb1_v5.cuh"
 #include "kb1_v6.cuh"
+#include "kb1_v9.cuh"
 #include "kb1_v8.cuh"
 #include "kb2_gather.cuh"
 #include "tables.h"
@@ -133,6 +134,16 @@ KB1Variant variant3v6() {
   using C = KB1V5Cfg<K>;
   return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v6<K, DIAG>, (const void *)&kb1_v6_3d<K, DIAG>, true, nullptr};
 }
+template <int K, int DIAG>
+void launch3v9(const KB1Args &a, int grid, cudaStream_t s) {
+  using C = KB1V5Cfg<K>;
+  kb1_v9_3d<K, DIAG><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+}
+template <int K, int DIAG = 0>
+KB1Variant variant3v9() {
+  using C = KB1V5Cfg<K>;
+  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v9<K, DIAG>, (const void *)&kb1_v9_3d<K, DIAG>, true, nullptr};
+}
 template <int K, int MINB>
 void launch3v8(const KB1Args &a, int grid, cudaStream_t s) {
   using C = KB1V8Cfg<K>;
@@ -165,9 +176,9 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
     switch (k) {
       case 1: add(variant3v2<1, 64, 2>(), "v2.z64"); add(variant3<1, 32, 2>(), "v1.z32"); break;
       case 2: add(variant3v2<2, 4, 3>(), "v2.z4"); add(variant3v3<2, 4, 2>(), "v3.z4"); add(variant3<2, 16, 2>(), "v1.z16"); break;
-      case 3: add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
+      case 3: add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
       case 4:
-        add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
+        add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v9<4>(), "v9"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
@@ -204,6 +215,8 @@ KB1Variant select_variant(int dim, int k) {
       if (strcmp(force, "v5.d2") == 0) { d = variant3v5<4, 2>(); d.name = "v5.d2"; return d; }
       if (strcmp(force, "v6.d1") == 0) { d = variant3v6<4, 1>(); d.name = "v6.d1"; return d; }
       if (strcmp(force, "v6.d2") == 0) { d = variant3v6<4, 2>(); d.name = "v6.d2"; return d; }
+      if (strcmp(force, "v9.d1") == 0) { d = variant3v9<4, 1>(); d.name = "v9.d1"; return d; }
+      if (strcmp(force, "v9.d2") == 0) { d = variant3v9<4, 2>(); d.name = "v9.d2"; return d; }
       if (strcmp(force, "v5.r2") == 0) { d = variant3v5<4, 0, 2>(); d.name = "v5.r2"; return d; }
       if (strcmp(force, "v5.r1d1") == 0) { d = variant3v5<4, 1, 1>(); d.name = "v5.r1d1"; return d; }
       if (strcmp(force, "v5.r2d1") == 0) { d = variant3v5<4, 1, 2>(); d.name = "v5.r2d1"; return d; }

@@ -85,6 +85,7 @@ __global__ void __launch_bounds__(KB1V2Cfg<K, ZPC>::NTH, MINB) kb1_v2_3d(const K
   constexpr int N = Dm::N, P = Dm::P, T = Dm::T, P2 = Dm::P2, P3 = Dm::P3, T2 = Dm::T2, T3 = Dm::T3;
   constexpr int N2 = Dm::N2, N3 = Dm::N3, TPZ = Dm::TPZ, NH = N / 2;
   constexpr int NTH = KB1V2Cfg<K, ZPC>::NTH;
+  static_assert(NTH <= 512, "block_min and the dt-filter slot share sRed[0, 32)");
   constexpr int IDS = KB1V2Cfg<K, ZPC>::IDS;
   extern __shared__ double smem[];
   double *sTab = smem;                               // B[N][P] G[N][P] Phi[N][T] W[N]
@@ -142,6 +143,7 @@ __global__ void __launch_bounds__(KB1V2Cfg<K, ZPC>::NTH, MINB) kb1_v2_3d(const K
   };
 
   for (int i = tid0; i < Dm::TAB; i += NTH) sTab[i] = __ldg(a.tab + i);
+  if (threadIdx.x == 0) sRed[16] = 0.0;   // dt filter: the CTA's best exact inverse dt (block_min uses sRed[0, 8))
   int64_t b = blockIdx.x;
   load_ids(b, tid0);
   issue(b, sPF, tid0);
@@ -291,7 +293,13 @@ __global__ void __launch_bounds__(KB1V2Cfg<K, ZPC>::NTH, MINB) kb1_v2_3d(const K
       const double R = active ? pfz[Dm::PF_R + q] : 1.0;
       const double alpha = sW[q0] * sW[q1] * sW[q2];
       PointOut<3> o;
-      point_eval3(Jm, Gv, eq, R, alpha, gamma, J0i, a.ph, o);
+      {   // dt filter (pointwise.cuh): exact sigma_min(J) only where a point can beat the CTA's best inverse dt
+        const unsigned vm = __activemask();
+        const double best = sRed[16];
+        point_eval3<true>(Jm, Gv, eq, R, alpha, gamma, J0i, a.ph, o, best, vm);
+        if (active && o.inv > best)
+          atomicMax(reinterpret_cast<unsigned long long *>(sRed + 16), (unsigned long long)__double_as_longlong(o.inv));
+      }
       if (h == 0) {
         double *SA = Rz + Dm::O_SA + (q2 * N + q1) * NH + q0a;
 #pragma unroll

@@ -62,6 +62,7 @@ __global__ void __launch_bounds__(KB1V3Cfg<K, ZPC>::NTH, MINB) kb1_v3_3d(const K
   constexpr int N = Dm::N, P = Dm::P, T = Dm::T, P2 = Dm::P2, P3 = Dm::P3, T2 = Dm::T2, T3 = Dm::T3;
   constexpr int N2 = Dm::N2, N3 = Dm::N3, TPZ = Dm::TPZ, NH = Dm::NH;
   constexpr int NTH = KB1V3Cfg<K, ZPC>::NTH, NW = KB1V3Cfg<K, ZPC>::NW;
+  static_assert(NTH <= 512, "block_min and the dt-filter slot share sRed[0, 32)");
   constexpr int MT_N = Dm::MT_N, MT_P = Dm::MT_P, MT_T = Dm::MT_T, KS_P = Dm::KS_P, KS_N = Dm::KS_N, KS_T = Dm::KS_T;
   extern __shared__ double smem[];
   double *sTab = smem;                                  // B[N][P] G[N][P] Phi[N][T] W[N]
@@ -83,6 +84,16 @@ __global__ void __launch_bounds__(KB1V3Cfg<K, ZPC>::NTH, MINB) kb1_v3_3d(const K
 
   // ---- a0: tables, gather ----------------------------------------------------------------------
   for (int i = tid; i < Dm::TAB; i += NTH) sTab[i] = __ldg(a.tab + i);
+  if (threadIdx.x == 0) sRed[16] = 0.0;   // dt filter: the CTA's best exact inverse dt (block_min uses sRed[0, 8))
+  {   // rho0|J0| of this thread's two points is read in the point stage: start the DRAM fetches into L1 now
+    const int zl = tid / Dm::TPZ, pr = tid - zl * Dm::TPZ;
+    if (zl < ZPC && zone0 + zl < Z) {
+      const int q = ((pr / (Dm::N / 2 * Dm::N)) * Dm::N + (pr / (Dm::N / 2)) % Dm::N) * Dm::N + pr % (Dm::N / 2);
+      const double *Rq = a.rho0detJ0 + (zone0 + zl) * Dm::N3 + q;
+      asm volatile("prefetch.global.L1 [%0];" ::"l"(Rq));
+      asm volatile("prefetch.global.L1 [%0];" ::"l"(Rq + Dm::N / 2));
+    }
+  }
   for (int i = tid; i < ZPC * P3; i += NTH) {
     const int zl = i / P3, r = i - zl * P3;
     const int64_t z = zone0 + zl;
@@ -265,7 +276,13 @@ __global__ void __launch_bounds__(KB1V3Cfg<K, ZPC>::NTH, MINB) kb1_v3_3d(const K
       const double R = active ? __ldg(a.rho0detJ0 + my_z * N3 + q) : 1.0;
       const double alpha = sW[q0] * sW[q1] * sW[q2];
       PointOut<3> o;
-      point_eval3(Jm, Gv, eq, R, alpha, gamma, J0i, a.ph, o);
+      {   // dt filter (pointwise.cuh): exact sigma_min(J) only where a point can beat the CTA's best inverse dt
+        const unsigned vm = __activemask();
+        const double best = sRed[16];
+        point_eval3<true>(Jm, Gv, eq, R, alpha, gamma, J0i, a.ph, o, best, vm);
+        if (active && o.inv > best)
+          atomicMax(reinterpret_cast<unsigned long long *>(sRed + 16), (unsigned long long)__double_as_longlong(o.inv));
+      }
       if (h == 0) {
         double *SA = Rz + Dm::O_SA + (q2 * N + q1) * NH + q0a;
 #pragma unroll

@@ -95,6 +95,10 @@ __global__ void __launch_bounds__(KB1V8Cfg<K>::NTH, MINB) kb1_v8_3d(const KB1Arg
 #pragma unroll 1
   for (int q2 = 0; q2 < N; ++q2) {
     const int o = a.zero * (q2 + 1);   // 0, but loop-variant and uniform: the table loads stay here
+    // rho0|J0| of this thread's point of slab q2 is read in the point stage: start its DRAM fetch into L1
+    // now, two stages ahead (ncu on v8: long_scoreboard was the second stall reason, profiles/r01_kb1_c5_default_ncu)
+    if (has_point)
+      asm volatile("prefetch.global.L1 [%0];" ::"l"(a.rho0detJ0 + z * (int64_t)(N * NS) + (q2 * N + q1) * N + q0));
     // ---- stage A: a2 -> q2 (TB, TG of the 6 fields; TE) -------------------------------------------
     {
       const CTZ<K> C{o};
