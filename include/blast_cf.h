@@ -105,7 +105,11 @@ int blast_cf_eval(blast_cf *h, const double *x, const double *v, const double *e
 
 /* Same evaluation with HOST buffers (pinned memory recommended): copies the inputs host->device,
  * evaluates, copies the three outputs back and synchronizes the stream before returning.  Device
- * staging buffers are allocated by the first call and reused. */
+ * staging buffers, two internal copy streams and the zone-chunk plan are created by the first call and
+ * reused.  On large meshes the copies overlap the computation chunk by chunk (zones in contiguous
+ * chunks; a chunk's corner force starts when its node prefix of x, v and its e, rho0detJ0 slices have
+ * arrived); the results are bitwise those of blast_cf_eval on the same data.  Errors: EINVAL for NULL
+ * arrays, ENOMEM / ECUDA as blast_cf_eval. */
 int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
                        double *out_Fdot1, double *out_FTv, double *out_dt_min);
 

@@ -22,7 +22,6 @@
 #include "kb1_v4.cuh"
 #include "kb1_v5.cuh"
 #include "kb1_v6.cuh"
-#include "kb1_v9.cuh"
 #include "kb1_v8.cuh"
 #include "kb2_gather.cuh"
 #include "tables.h"
@@ -81,16 +80,16 @@ void launch2(const KB1Args &a, int grid, cudaStream_t s) {
   using C = KB1Cfg2<K, ZPC>;
   kb1_corner_force_2d<K, ZPC, MINB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
 }
-template <int K, int ZPC, int MINB>
+template <int K, int ZPC, int MINB, int PPT>
 void launch3v2(const KB1Args &a, int grid, cudaStream_t s) {
-  using C = KB1V2Cfg<K, ZPC>;
-  kb1_v2_3d<K, ZPC, MINB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+  using C = KB1V2Cfg<K, ZPC, PPT>;
+  kb1_v2_3d<K, ZPC, MINB, PPT><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
 }
-template <int K, int ZPC, int MINB>
+template <int K, int ZPC, int MINB, int PPT = 2>
 KB1Variant variant3v2() {
-  using C = KB1V2Cfg<K, ZPC>;
-  return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3v2<K, ZPC, MINB>, (const void *)&kb1_v2_3d<K, ZPC, MINB>,
-                    true, nullptr};
+  using C = KB1V2Cfg<K, ZPC, PPT>;
+  return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3v2<K, ZPC, MINB, PPT>,
+                    (const void *)&kb1_v2_3d<K, ZPC, MINB, PPT>, true, nullptr};
 }
 template <int K, int ZPC, int MINB>
 void launch3v3(const KB1Args &a, int grid, cudaStream_t s) {
@@ -134,16 +133,6 @@ KB1Variant variant3v6() {
   using C = KB1V5Cfg<K>;
   return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v6<K, DIAG>, (const void *)&kb1_v6_3d<K, DIAG>, true, nullptr};
 }
-template <int K, int DIAG>
-void launch3v9(const KB1Args &a, int grid, cudaStream_t s) {
-  using C = KB1V5Cfg<K>;
-  kb1_v9_3d<K, DIAG><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
-}
-template <int K, int DIAG = 0>
-KB1Variant variant3v9() {
-  using C = KB1V5Cfg<K>;
-  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v9<K, DIAG>, (const void *)&kb1_v9_3d<K, DIAG>, true, nullptr};
-}
 template <int K, int MINB>
 void launch3v8(const KB1Args &a, int grid, cudaStream_t s) {
   using C = KB1V8Cfg<K>;
@@ -174,11 +163,11 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
   auto add = [&](KB1Variant x, const char *name) { x.name = name; v.push_back(x); };
   if (dim == 3) {
     switch (k) {
-      case 1: add(variant3v2<1, 64, 2>(), "v2.z64"); add(variant3<1, 32, 2>(), "v1.z32"); break;
-      case 2: add(variant3v2<2, 4, 3>(), "v2.z4"); add(variant3v3<2, 4, 2>(), "v3.z4"); add(variant3<2, 16, 2>(), "v1.z16"); break;
-      case 3: add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
+      case 1: add(variant3v2<1, 32, 2, 1>(), "v2.p1.z32"); add(variant3v2<1, 64, 2>(), "v2.z64"); add(variant3<1, 32, 2>(), "v1.z32"); break;
+      case 2: add(variant3v2<2, 4, 3>(), "v2.z4"); add(variant3v2<2, 4, 2, 1>(), "v2.p1.z4"); add(variant3v2<2, 2, 4, 1>(), "v2.p1.z2"); add(variant3v3<2, 4, 2>(), "v3.z4"); add(variant3<2, 16, 2>(), "v1.z16"); break;
+      case 3: add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3v2<3, 1, 2, 1>(), "v2.p1.z1"); add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
       case 4:
-        add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v9<4>(), "v9"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
+        add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
@@ -215,8 +204,6 @@ KB1Variant select_variant(int dim, int k) {
       if (strcmp(force, "v5.d2") == 0) { d = variant3v5<4, 2>(); d.name = "v5.d2"; return d; }
       if (strcmp(force, "v6.d1") == 0) { d = variant3v6<4, 1>(); d.name = "v6.d1"; return d; }
       if (strcmp(force, "v6.d2") == 0) { d = variant3v6<4, 2>(); d.name = "v6.d2"; return d; }
-      if (strcmp(force, "v9.d1") == 0) { d = variant3v9<4, 1>(); d.name = "v9.d1"; return d; }
-      if (strcmp(force, "v9.d2") == 0) { d = variant3v9<4, 2>(); d.name = "v9.d2"; return d; }
       if (strcmp(force, "v5.r2") == 0) { d = variant3v5<4, 0, 2>(); d.name = "v5.r2"; return d; }
       if (strcmp(force, "v5.r1d1") == 0) { d = variant3v5<4, 1, 1>(); d.name = "v5.r1d1"; return d; }
       if (strcmp(force, "v5.r2d1") == 0) { d = variant3v5<4, 1, 2>(); d.name = "v5.r2d1"; return d; }
@@ -392,8 +379,19 @@ struct blast_cf {
   // device memory
   double *d_tab = nullptr, *d_J0inv = nullptr, *d_gamma = nullptr, *d_Fz1 = nullptr, *d_ctadt = nullptr;
   int32_t *d_zone_nodes = nullptr, *d_ptr = nullptr, *d_ent = nullptr;
-  // host-eval staging
+  // host-eval staging (blast_cf_eval_host): device copies of the inputs/outputs and the zone-chunk pipeline
   double *d_in = nullptr, *d_out = nullptr;
+  struct HostPipe {
+    static constexpr int MAXC = 8;
+    const void *plan_for = nullptr;          // KB1 function the plan was built for (autotune may switch it)
+    int nch = 0;                             // zone chunks (1 = no pipelining)
+    int64_t z0[MAXC + 1] = {};               // chunk c = zones [z0[c], z0[c+1])
+    int64_t hi[MAXC] = {};                   // max node id over the zones of chunks 0..c (prefix max)
+    int grid[MAXC] = {}, off[MAXC] = {}, nslots = 0;   // KB1 grid and per-CTA dt slots of each chunk
+    double *d_ctadt = nullptr;
+    cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
+    cudaEvent_t ev_in[MAXC] = {}, ev_kb1[MAXC] = {}, ev_d2h = nullptr, ev_start = nullptr;
+  } hp;
   long long *d_prof = nullptr;   // stage timestamps (BLAST_CF_PROFILE=1)
   // timing
   bool timing = false;
@@ -411,6 +409,15 @@ void free_handle(blast_cf *h) {
   for (auto &e : h->ev)
     if (e) cudaEventDestroy(e);
   if (h->xch) blastcf::exchange_destroy(h->xch);
+  cudaFree(h->hp.d_ctadt);
+  for (int c = 0; c < blast_cf::HostPipe::MAXC; ++c) {
+    if (h->hp.ev_in[c]) cudaEventDestroy(h->hp.ev_in[c]);
+    if (h->hp.ev_kb1[c]) cudaEventDestroy(h->hp.ev_kb1[c]);
+  }
+  if (h->hp.ev_d2h) cudaEventDestroy(h->hp.ev_d2h);
+  if (h->hp.ev_start) cudaEventDestroy(h->hp.ev_start);
+  if (h->hp.s_h2d) cudaStreamDestroy(h->hp.s_h2d);
+  if (h->hp.s_d2h) cudaStreamDestroy(h->hp.s_d2h);
   delete h;
 }
 
@@ -707,27 +714,141 @@ int blast_cf_eval(blast_cf *h, const double *x, const double *v, const double *e
   return eval_impl(h, x, v, e, rho0detJ0, out_Fdot1, out_FTv, out_dt_min, nullptr);
 }
 
+// The host-buffer entry overlaps the PCIe transfers with the corner force: the zones are split into up
+// to 8 contiguous chunks; chunk c's KB1 starts as soon as its inputs are on the device (the node prefix
+// [0, hi[c]] of x and v, its e and rho0|J0| slices, copied on a second stream), its F^T v slice goes back
+// on a third stream while later chunks compute, and KB2 + the F.1 copy follow the last chunk.  Each chunk's
+// KB1 is the same kernel on a zone sub-range (shifted zone-indexed pointers), with its own per-CTA dt slots.
+static int host_plan(blast_cf *h) {
+  blast_cf::HostPipe &P = h->hp;
+  if (P.plan_for == h->var.func) return BLAST_CF_OK;
+  // zones one wave of resident CTAs covers: the persistent grid, else occupancy x SMs
+  int resident = h->ncta;
+  if (!h->var.persistent) {
+    int occ = 0, sms = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, h->var.func, h->var.nth, h->var.smem);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device);
+    resident = std::max(1, occ) * std::max(1, sms);
+  }
+  const int64_t per_wave = (int64_t)std::max(resident, 1) * std::max(h->var.zpc, 1);
+  int nch = (int)std::min<int64_t>(blast_cf::HostPipe::MAXC, h->Z / (2 * per_wave));
+  if (h->xch) nch = 1;   // multi-rank: keep the plain path (the exchange follows KB2 anyway)
+  nch = std::max(nch, 1);
+  std::vector<int32_t> zn((size_t)h->Z * h->nk);
+  if (nch > 1) CUDA_TRY(cudaMemcpy(zn.data(), h->d_zone_nodes, zn.size() * sizeof(int32_t), cudaMemcpyDeviceToHost));
+  P.nch = nch;
+  P.nslots = 0;
+  int64_t hi = -1;
+  for (int c = 0; c < nch; ++c) {
+    P.z0[c] = h->Z * c / nch;
+    P.z0[c + 1] = h->Z * (c + 1) / nch;
+    for (size_t i = (size_t)P.z0[c] * h->nk; nch > 1 && i < (size_t)P.z0[c + 1] * h->nk; ++i) hi = std::max<int64_t>(hi, zn[i]);
+    P.hi[c] = nch > 1 ? hi : h->nn - 1;
+    const int64_t zc = P.z0[c + 1] - P.z0[c];
+    int g = (int)((zc + h->var.zpc - 1) / h->var.zpc);
+    if (h->var.persistent) g = std::min(g, h->ncta);
+    P.grid[c] = g;
+    P.off[c] = P.nslots;
+    P.nslots += g;
+  }
+  cudaFree(P.d_ctadt);
+  P.d_ctadt = nullptr;
+  CUDA_TRY(cudaMalloc(&P.d_ctadt, std::max(P.nslots, 1) * sizeof(double)));
+  if (!P.s_h2d) {
+    CUDA_TRY(cudaStreamCreateWithFlags(&P.s_h2d, cudaStreamNonBlocking));
+    CUDA_TRY(cudaStreamCreateWithFlags(&P.s_d2h, cudaStreamNonBlocking));
+    for (int c = 0; c < blast_cf::HostPipe::MAXC; ++c) {
+      CUDA_TRY(cudaEventCreateWithFlags(&P.ev_in[c], cudaEventDisableTiming));
+      CUDA_TRY(cudaEventCreateWithFlags(&P.ev_kb1[c], cudaEventDisableTiming));
+    }
+    CUDA_TRY(cudaEventCreateWithFlags(&P.ev_d2h, cudaEventDisableTiming));
+    CUDA_TRY(cudaEventCreateWithFlags(&P.ev_start, cudaEventDisableTiming));
+  }
+  P.plan_for = h->var.func;
+  return BLAST_CF_OK;
+}
+
 int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
                        double *out_Fdot1, double *out_FTv, double *out_dt_min) {
   if (!h) return fail(BLAST_CF_EINVAL, "handle is NULL");
+  if (!out_dt_min || ((!x || !v || !out_Fdot1) && h->nn > 0) || ((!e || !rho0detJ0 || !out_FTv) && h->Z > 0))
+    return fail(BLAST_CF_EINVAL, "NULL array argument");
+  int rc = check_async(h);
+  if (rc) return rc;
   const size_t nx = (size_t)h->dim * h->nn, ne = (size_t)h->Z * h->nt, nr = (size_t)h->Z * h->nq;
   if (!h->d_in) {
     CUDA_TRY(cudaMalloc(&h->d_in, (2 * nx + ne + nr + 1) * sizeof(double)));
     CUDA_TRY(cudaMalloc(&h->d_out, (nx + ne + 1) * sizeof(double)));
   }
+  if ((rc = host_plan(h))) return rc;
+  blast_cf::HostPipe &P = h->hp;
   double *dx = h->d_in, *dv = dx + nx, *de = dv + nx, *dr = de + ne;
   double *dF = h->d_out, *dT = dF + nx, *dd = dT + ne;
-  CUDA_TRY(cudaMemcpyAsync(dx, x, nx * sizeof(double), cudaMemcpyHostToDevice, h->stream));
-  CUDA_TRY(cudaMemcpyAsync(dv, v, nx * sizeof(double), cudaMemcpyHostToDevice, h->stream));
-  CUDA_TRY(cudaMemcpyAsync(de, e, ne * sizeof(double), cudaMemcpyHostToDevice, h->stream));
-  CUDA_TRY(cudaMemcpyAsync(dr, rho0detJ0, nr * sizeof(double), cudaMemcpyHostToDevice, h->stream));
-  int rc = blast_cf_eval(h, dx, dv, de, dr, dF, dT, dd);
-  if (rc) return rc;
+  if (P.nch == 1 || h->timing || h->d_prof) {   // plain path: copy in, evaluate, copy out
+    CUDA_TRY(cudaMemcpyAsync(dx, x, nx * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(cudaMemcpyAsync(dv, v, nx * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(cudaMemcpyAsync(de, e, ne * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+    CUDA_TRY(cudaMemcpyAsync(dr, rho0detJ0, nr * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+    if ((rc = blast_cf_eval(h, dx, dv, de, dr, dF, dT, dd))) return rc;
+    CUDA_TRY(cudaMemcpyAsync(out_Fdot1, dF, nx * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaMemcpyAsync(out_FTv, dT, ne * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaMemcpyAsync(out_dt_min, dd, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+    CUDA_TRY(cudaStreamSynchronize(h->stream));
+    return BLAST_CF_OK;
+  }
+  // the copy streams start after everything already queued on the handle's stream
+  CUDA_TRY(cudaEventRecord(P.ev_start, h->stream));
+  CUDA_TRY(cudaStreamWaitEvent(P.s_h2d, P.ev_start, 0));
+  CUDA_TRY(cudaStreamWaitEvent(P.s_d2h, P.ev_start, 0));
+  KB1Args a;
+  a.zone_nodes = h->d_zone_nodes; a.J0inv = h->d_J0inv; a.zone_gamma = h->d_gamma; a.tab = h->d_tab;
+  a.x = dx; a.v = dv; a.e = de; a.rho0detJ0 = dr; a.Fz1 = h->d_Fz1; a.FTv = dT; a.cta_dt = P.d_ctadt;
+  a.Sq = nullptr; a.prof = nullptr; a.num_nodes = h->nn; a.zero = 0;
+  a.ph.cfl = h->params.cfl; a.ph.q_quad = h->params.q_quad; a.ph.q_lin = h->params.q_lin;
+  a.ph.eps_sw = h->params.eps_switch; a.ph.inv_2eps = 0.5 / h->params.eps_switch; a.ph.h0 = h->h0; a.ph.k = (double)h->k;
+  a.ph.use_visc = h->params.use_viscosity; a.ph.use_vort = h->params.use_vorticity;
+  int64_t done = 0;   // nodes [0, done) of x and v are on their way
+  for (int c = 0; c < P.nch; ++c) {
+    const int64_t z0 = P.z0[c], zc = P.z0[c + 1] - z0, n1 = P.hi[c] + 1;
+    if (n1 > done) {
+      for (int d = 0; d < h->dim; ++d) {
+        CUDA_TRY(cudaMemcpyAsync(dx + d * h->nn + done, x + d * h->nn + done, (n1 - done) * sizeof(double),
+                                 cudaMemcpyHostToDevice, P.s_h2d));
+        CUDA_TRY(cudaMemcpyAsync(dv + d * h->nn + done, v + d * h->nn + done, (n1 - done) * sizeof(double),
+                                 cudaMemcpyHostToDevice, P.s_h2d));
+      }
+      done = n1;
+    }
+    CUDA_TRY(cudaMemcpyAsync(de + z0 * h->nt, e + z0 * h->nt, zc * h->nt * sizeof(double), cudaMemcpyHostToDevice, P.s_h2d));
+    CUDA_TRY(cudaMemcpyAsync(dr + z0 * h->nq, rho0detJ0 + z0 * h->nq, zc * h->nq * sizeof(double),
+                             cudaMemcpyHostToDevice, P.s_h2d));
+    CUDA_TRY(cudaEventRecord(P.ev_in[c], P.s_h2d));
+    CUDA_TRY(cudaStreamWaitEvent(h->stream, P.ev_in[c], 0));
+    KB1Args ac = a;   // the same kernel on zones [z0, z0 + zc): zone-indexed arrays shifted
+    ac.zone_nodes = h->d_zone_nodes + z0 * h->nk; ac.J0inv = h->d_J0inv + z0 * 9; ac.zone_gamma = h->d_gamma + z0;
+    ac.e = de + z0 * h->nt; ac.rho0detJ0 = dr + z0 * h->nq; ac.Fz1 = h->d_Fz1 + z0 * h->dim * h->nk;
+    ac.FTv = dT + z0 * h->nt; ac.cta_dt = P.d_ctadt + P.off[c]; ac.num_zones = zc;
+    if (P.grid[c] > 0) h->var.launch(ac, P.grid[c], h->stream);
+    CUDA_TRY(cudaEventRecord(P.ev_kb1[c], h->stream));
+    CUDA_TRY(cudaStreamWaitEvent(P.s_d2h, P.ev_kb1[c], 0));
+    CUDA_TRY(cudaMemcpyAsync(out_FTv + z0 * h->nt, dT + z0 * h->nt, zc * h->nt * sizeof(double), cudaMemcpyDeviceToHost,
+                             P.s_d2h));
+  }
+  // (nodes above hi[nch-1] belong to no zone: KB2 gives them F.1 = 0 without reading x or v)
+  const int gthreads = 256;
+  const int64_t gblocks = std::max<int64_t>(1, (h->nn + gthreads - 1) / gthreads);
+  if (h->dim == 3)
+    kb2_gather<3, 8><<<(unsigned)gblocks, gthreads, 0, h->stream>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->nk, dF,
+                                                                     P.d_ctadt, P.nslots, dd);
+  else
+    kb2_gather<2, 4><<<(unsigned)gblocks, gthreads, 0, h->stream>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->nk, dF,
+                                                                     P.d_ctadt, P.nslots, dd);
   CUDA_TRY(cudaMemcpyAsync(out_Fdot1, dF, nx * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
-  CUDA_TRY(cudaMemcpyAsync(out_FTv, dT, ne * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
   CUDA_TRY(cudaMemcpyAsync(out_dt_min, dd, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+  CUDA_TRY(cudaEventRecord(P.ev_d2h, P.s_d2h));
+  CUDA_TRY(cudaStreamWaitEvent(h->stream, P.ev_d2h, 0));
   CUDA_TRY(cudaStreamSynchronize(h->stream));
-  return BLAST_CF_OK;
+  return check_async(h);
 }
 
 int blast_cf_eval_debug_Fz(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,

@@ -57,10 +57,12 @@ struct V2Dims {
   static constexpr int TAB = 2 * N * P + N * T + N;   // per-thread-indexed table copy (stage C)
 };
 
-template <int K, int ZPC>
+// PPT = quadrature points per thread: 2 (q0 and q0 + N/2 in turn) or 1 (twice the threads, fewer registers)
+template <int K, int ZPC, int PPT = 2>
 struct KB1V2Cfg {
   using Dm = V2Dims<K>;
-  static constexpr int NTH = (ZPC * Dm::TPZ + 31) / 32 * 32;
+  static constexpr int TPZ = Dm::N3 / PPT;                // threads per zone
+  static constexpr int NTH = (ZPC * TPZ + 31) / 32 * 32;
   static constexpr int SMEM_DOUBLES = (Dm::TAB + 1) / 2 * 2 + 2 * ZPC * Dm::PFZ + ZPC * Dm::ZONE + 32;
   static constexpr int SMEM_BYTES = SMEM_DOUBLES * 8;
   static constexpr int IDS = (ZPC * Dm::P3 + NTH - 1) / NTH;   // node ids a thread prefetches per batch
@@ -78,15 +80,17 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int NPEND>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(NPEND)); }
 
-template <int K, int ZPC, int MINB>
-__global__ void __launch_bounds__(KB1V2Cfg<K, ZPC>::NTH, MINB) kb1_v2_3d(const KB1Args a) {
+template <int K, int ZPC, int MINB, int PPT = 2>
+__global__ void __launch_bounds__(KB1V2Cfg<K, ZPC, PPT>::NTH, MINB) kb1_v2_3d(const KB1Args a) {
   using Dm = V2Dims<K>;
   using C = CT<K>;
   constexpr int N = Dm::N, P = Dm::P, T = Dm::T, P2 = Dm::P2, P3 = Dm::P3, T2 = Dm::T2, T3 = Dm::T3;
-  constexpr int N2 = Dm::N2, N3 = Dm::N3, TPZ = Dm::TPZ, NH = N / 2;
-  constexpr int NTH = KB1V2Cfg<K, ZPC>::NTH;
+  constexpr int N2 = Dm::N2, N3 = Dm::N3, NH = N / 2;
+  constexpr int TPZ = KB1V2Cfg<K, ZPC, PPT>::TPZ;
+  constexpr int NTH = KB1V2Cfg<K, ZPC, PPT>::NTH;
+  static_assert(PPT == 1 || PPT == 2, "kb1_v2: one or two points per thread");
   static_assert(NTH <= 512, "block_min and the dt-filter slot share sRed[0, 32)");
-  constexpr int IDS = KB1V2Cfg<K, ZPC>::IDS;
+  constexpr int IDS = KB1V2Cfg<K, ZPC, PPT>::IDS;
   extern __shared__ double smem[];
   double *sTab = smem;                               // B[N][P] G[N][P] Phi[N][T] W[N]
   double *sPF = smem + (Dm::TAB + 1) / 2 * 2;        // [2][ZPC][PFZ]
@@ -257,7 +261,9 @@ __global__ void __launch_bounds__(KB1V2Cfg<K, ZPC>::NTH, MINB) kb1_v2_3d(const K
   const bool has_point = my_zl < ZPC;
   const int64_t my_z = zone0 + my_zl;
   const bool active = has_point && my_z < Z;
-  const int q0a = pr % NH, q1 = (pr / NH) % N, q2 = pr / (NH * N);
+  // PPT 2: points (q0a, q1, q2) and (q0a + N/2, q1, q2);  PPT 1: the point (q0a + hsel N/2, q1, q2)
+  const int q0a = PPT == 2 ? pr % NH : (pr % N) % NH, hsel = PPT == 2 ? 0 : (pr % N) / NH;
+  const int q1 = PPT == 2 ? (pr / NH) % N : (pr / N) % N, q2 = PPT == 2 ? pr / (NH * N) : pr / N2;
   double SB[10];
   if (has_point) {
     double *Rz = sZone + my_zl * Dm::ZONE;
@@ -267,7 +273,8 @@ __global__ void __launch_bounds__(KB1V2Cfg<K, ZPC>::NTH, MINB) kb1_v2_3d(const K
     const double gamma = J0i[9];
     const double *sW = sTab + 2 * N * P + N * T;
 #pragma unroll 1
-    for (int h = 0; h < 2; ++h) {
+    for (int hh = 0; hh < PPT; ++hh) {
+      const int h = PPT == 2 ? hh : hsel;
       const int q0 = q0a + h * NH;
       double g[18];
 #pragma unroll
@@ -321,7 +328,7 @@ __global__ void __launch_bounds__(KB1V2Cfg<K, ZPC>::NTH, MINB) kb1_v2_3d(const K
     }
   }
   __syncthreads();   // every U read is done
-  if (has_point) {
+  if (has_point && (PPT == 2 || hsel == 1)) {
     double *SBp = sZone + my_zl * Dm::ZONE + Dm::R0 + Dm::O_SB + (q2 * N + q1) * NH + q0a;
 #pragma unroll
     for (int cd = 0; cd < 10; ++cd) SBp[cd * N2 * NH] = SB[cd];

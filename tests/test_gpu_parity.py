@@ -134,6 +134,19 @@ def test_eval_host_matches_device():
     assert np.array_equal(o[0], F1) and np.array_equal(o[1], FTv) and o[2][0] == dt
 
 
+@pytest.mark.parametrize("name", ["C3", "C4", "C5"])
+def test_eval_host_pipelined_matches_device(name):
+    """At full size the host entry splits the zones into chunks whose copies overlap the kernels (a KB1
+    launch per zone sub-range, per-chunk dt slots): every output must equal the device entry's bit for bit."""
+    torch = _torch()
+    m, s = synth.config(name, "S1")
+    h, [(F1, FTv, dt)] = gpu_eval(m, s)
+    hx = [torch.from_numpy(np.ascontiguousarray(a)).pin_memory() for a in (s.x, s.v, s.e, s.rho0detJ0)]
+    for _ in range(2):   # twice: the second call reuses the plan and the staging buffers
+        o = h.eval_host(*hx)
+        assert np.array_equal(o[0], F1) and np.array_equal(o[1], FTv) and o[2][0] == dt
+
+
 @pytest.mark.parametrize("name,N,k", [("C1", None, None), ("C3", (2, 2, 1), None), ("C2", (2, 2), 3)])
 def test_debug_Fz_matches_oracle_definition_mode(orc, name, N, k):
     torch = _torch()
@@ -199,6 +212,14 @@ def test_full_size_sampled(orc, name, which):
     sampled_parity(orc, name, which, n_nodes=24 if name == "C5" else 48, n_zones=8 if name == "C5" else 48)
 
 
+@pytest.mark.parametrize("name", ["v6", "v4.m0"])
+def test_full_size_sampled_c4_variants(orc, name, monkeypatch):
+    """The persistent warp-specialized C4 candidates at the bench's size (221 zones per CTA: every stage of
+    the zone pipeline, both buffers and the dt filter across zones are exercised)."""
+    monkeypatch.setenv("BLAST_CF_KB1", name)
+    sampled_parity(orc, "C4", "S1")
+
+
 def test_non_affine_initial_mesh(orc):
     """Reading R19: the GPU keeps J0^{-1} per zone, so a curved initial mesh is rejected when the
     viscosity (which needs J0) is on, and evaluated normally when it is off."""
@@ -221,7 +242,8 @@ def test_multi_material_gamma(orc):
     check(m, s, orc)
 
 
-CANDIDATES = {2: ["v2.z4", "v3.z4", "v1.z16"], 3: ["v3.z2", "v2.z2", "v1.z8"],
+CANDIDATES = {1: ["v2.p1.z32", "v2.z64", "v1.z32"], 2: ["v2.z4", "v2.p1.z4", "v2.p1.z2", "v3.z4", "v1.z16"],
+              3: ["v2.z2", "v2.p1.z1", "v3.z2", "v1.z8"],
               4: ["v5.r1", "v4.m0", "v5", "v6", "v4.m1", "v3.z1", "v2.z1", "v1.z4"],
               7: ["v8", "v1.z1"], 8: ["v8", "v8.m1", "v1.z1m2", "v1.z1"]}
 
