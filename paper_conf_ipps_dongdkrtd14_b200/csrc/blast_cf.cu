@@ -22,6 +22,7 @@
 #include "kb1_v4.cuh"
 #include "kb1_v5.cuh"
 #include "kb1_v6.cuh"
+#include "kb1_v10.cuh"
 #include "kb1_v8.cuh"
 #include "kb2_gather.cuh"
 #include "tables.h"
@@ -133,6 +134,17 @@ KB1Variant variant3v6() {
   using C = KB1V5Cfg<K>;
   return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v6<K, DIAG>, (const void *)&kb1_v6_3d<K, DIAG>, true, nullptr};
 }
+template <int K, int DIAG, int MODE, int OPT>
+void launch3v10(const KB1Args &a, int grid, cudaStream_t s) {
+  using C = KB1V5Cfg<K, MODE>;
+  kb1_v10_3d<K, DIAG, MODE, OPT><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+}
+template <int K, int DIAG = 0, int MODE = 0, int OPT = 0>
+KB1Variant variant3v10() {
+  using C = KB1V5Cfg<K, MODE>;
+  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v10<K, DIAG, MODE, OPT>,
+                    (const void *)&kb1_v10_3d<K, DIAG, MODE, OPT>, true, nullptr};
+}
 template <int K, int MINB>
 void launch3v8(const KB1Args &a, int grid, cudaStream_t s) {
   using C = KB1V8Cfg<K>;
@@ -167,7 +179,7 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
       case 2: add(variant3v2<2, 4, 3>(), "v2.z4"); add(variant3v2<2, 4, 2, 1>(), "v2.p1.z4"); add(variant3v2<2, 2, 4, 1>(), "v2.p1.z2"); add(variant3v3<2, 4, 2>(), "v3.z4"); add(variant3<2, 16, 2>(), "v1.z16"); break;
       case 3: add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3v2<3, 1, 2, 1>(), "v2.p1.z1"); add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
       case 4:
-        add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
+        add(variant3v10<4>(), "v10"); add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
@@ -204,6 +216,11 @@ KB1Variant select_variant(int dim, int k) {
       if (strcmp(force, "v5.d2") == 0) { d = variant3v5<4, 2>(); d.name = "v5.d2"; return d; }
       if (strcmp(force, "v6.d1") == 0) { d = variant3v6<4, 1>(); d.name = "v6.d1"; return d; }
       if (strcmp(force, "v6.d2") == 0) { d = variant3v6<4, 2>(); d.name = "v6.d2"; return d; }
+      if (strcmp(force, "v10.q") == 0) { d = variant3v10<4, 0, 0, 4>(); d.name = "v10.q"; return d; }
+      if (strcmp(force, "v10.b") == 0) { d = variant3v10<4, 0, 0, 1>(); d.name = "v10.b"; return d; }
+      if (strcmp(force, "v10.l") == 0) { d = variant3v10<4, 0, 0, 2>(); d.name = "v10.l"; return d; }
+      if (strcmp(force, "v10.d1") == 0) { d = variant3v10<4, 1>(); d.name = "v10.d1"; return d; }
+      if (strcmp(force, "v10.d2") == 0) { d = variant3v10<4, 2>(); d.name = "v10.d2"; return d; }
       if (strcmp(force, "v5.r2") == 0) { d = variant3v5<4, 0, 2>(); d.name = "v5.r2"; return d; }
       if (strcmp(force, "v5.r1d1") == 0) { d = variant3v5<4, 1, 1>(); d.name = "v5.r1d1"; return d; }
       if (strcmp(force, "v5.r2d1") == 0) { d = variant3v5<4, 1, 2>(); d.name = "v5.r2d1"; return d; }
@@ -289,6 +306,7 @@ int exchange_create(Exchange **out, const blast_cf_mesh *mesh, int dim, int64_t 
   x->num_nbr = mesh->num_neighbors; x->stream = stream; x->nrows = total;
   x->nbr_rank.assign(mesh->nbr_rank, mesh->nbr_rank + x->num_nbr);
   x->nbr_offset.assign(mesh->nbr_offset, mesh->nbr_offset + x->num_nbr + 1);
+  x->h_rows.assign(mesh->nbr_nodes, mesh->nbr_nodes + total);
   ExchangePlan pl = build_plan(x->rank, x->num_nbr, mesh->nbr_rank, mesh->nbr_offset, mesh->nbr_nodes);
   x->nu = (int64_t)pl.unique_nodes.size();
   int rc;
@@ -695,6 +713,9 @@ int handle_view(const blast_cf *h, HandleView *o) {
   o->Z = h->Z; o->nn = h->nn; o->stream = h->stream; o->device = h->device;
   o->zone_nodes = h->d_zone_nodes; o->ptr = h->d_ptr; o->ent = h->d_ent; o->tab = h->d_tab;
   o->multi_rank = h->xch != nullptr;
+  o->rank = h->xch ? h->xch->rank : 0;
+  o->nranks = h->xch ? h->xch->nranks : 1;
+  o->loopback = h->xch != nullptr && h->xch->comm == nullptr;
   return BLAST_CF_OK;
 }
 
@@ -704,6 +725,99 @@ int eval_with_S(blast_cf *h, const double *x, const double *v, const double *e, 
 }
 
 int set_error(int code, const char *msg) { return fail(code, "%s", msg); }
+
+// a loopback group: hs[r] is rank r of an n-rank decomposition without a communicator
+static int check_group(blast_cf *const *hs, int n, bool *loop) {
+  if (!hs || n < 1 || !hs[0]) return fail(BLAST_CF_EINVAL, "NULL group");
+  *loop = hs[0]->xch && !hs[0]->xch->comm;
+  if (!*loop) return n == 1 ? BLAST_CF_OK : fail(BLAST_CF_EINVAL, "an NCCL group call drives one rank (n = 1)");
+  for (int r = 0; r < n; ++r)
+    if (!hs[r] || !hs[r]->xch || hs[r]->xch->comm || hs[r]->xch->nranks != n || hs[r]->xch->rank != r)
+      return fail(BLAST_CF_EINVAL, "handle %d is not rank %d of a %d-rank loopback group", r, r, n);
+  return BLAST_CF_OK;
+}
+
+// rank r's recv rows from q are rank q's send rows for r (same order: global node id)
+static int loopback_move(blast_cf *const *hs, int n) {
+  for (int r = 0; r < n; ++r) CUDA_TRY(cudaStreamSynchronize(hs[r]->stream));
+  for (int r = 0; r < n; ++r) {
+    Exchange *xr = hs[r]->xch;
+    for (int i = 0; i < xr->num_nbr; ++i) {
+      const int q = xr->nbr_rank[i];
+      Exchange *xq = hs[q]->xch;
+      int iq = -1;
+      for (int t = 0; t < xq->num_nbr; ++t)
+        if (xq->nbr_rank[t] == r) iq = t;
+      const int64_t cnt = xr->nbr_offset[i + 1] - xr->nbr_offset[i];
+      if (iq < 0 || xq->nbr_offset[iq + 1] - xq->nbr_offset[iq] != cnt)
+        return fail(BLAST_CF_EINVAL, "ranks %d and %d disagree on their shared nodes", r, q);
+      CUDA_TRY(cudaMemcpy(xr->d_recv + xr->nbr_offset[i] * xr->dim, xq->d_send + xq->nbr_offset[iq] * xq->dim,
+                          cnt * xr->dim * sizeof(double), cudaMemcpyDeviceToDevice));
+    }
+  }
+  return BLAST_CF_OK;
+}
+
+int group_exchange_sum(blast_cf *const *hs, int n, double *const *vec) {
+  bool loop = false;
+  int rc = check_group(hs, n, &loop);
+  if (rc) return rc;
+  if (!hs[0]->xch) return BLAST_CF_OK;   // single rank: nothing is shared
+  if (!loop) {
+    Exchange *x = hs[0]->xch;
+    const int dim = x->dim;
+    exchange_pack(x, vec[0]);
+    NCCL_TRY(x->api->GroupStart(), "ncclGroupStart");
+    for (int i = 0; i < x->num_nbr; ++i) {
+      const int64_t o = x->nbr_offset[i], cnt = x->nbr_offset[i + 1] - o;
+      if (cnt == 0) continue;
+      NCCL_TRY(x->api->Send(x->d_send + o * dim, (size_t)cnt * dim, ncclDouble, x->nbr_rank[i], x->comm, x->stream), "ncclSend");
+      NCCL_TRY(x->api->Recv(x->d_recv + o * dim, (size_t)cnt * dim, ncclDouble, x->nbr_rank[i], x->comm, x->stream), "ncclRecv");
+    }
+    NCCL_TRY(x->api->GroupEnd(), "ncclGroupEnd");
+    exchange_combine(x, vec[0]);
+    return BLAST_CF_OK;
+  }
+  for (int r = 0; r < n; ++r) exchange_pack(hs[r]->xch, vec[r]);
+  if ((rc = loopback_move(hs, n))) return rc;
+  for (int r = 0; r < n; ++r) exchange_combine(hs[r]->xch, vec[r]);
+  return BLAST_CF_OK;
+}
+
+int group_allreduce(blast_cf *const *hs, int n, double *const *buf, int count, int op) {
+  bool loop = false;
+  int rc = check_group(hs, n, &loop);
+  if (rc) return rc;
+  if (!hs[0]->xch || count <= 0) return BLAST_CF_OK;
+  if (!loop) {
+    Exchange *x = hs[0]->xch;
+    const ncclRedOp_t o = op == 0 ? ncclSum : op == 1 ? ncclMin : ncclMax;
+    NCCL_TRY(x->api->AllReduce(buf[0], buf[0], (size_t)count, ncclDouble, o, x->comm, x->stream), "ncclAllReduce");
+    return BLAST_CF_OK;
+  }
+  std::vector<double> acc((size_t)count), part((size_t)count);
+  for (int r = 0; r < n; ++r) {   // ascending rank order
+    CUDA_TRY(cudaMemcpyAsync(part.data(), buf[r], count * sizeof(double), cudaMemcpyDeviceToHost, hs[r]->stream));
+    CUDA_TRY(cudaStreamSynchronize(hs[r]->stream));
+    for (int i = 0; i < count; ++i)
+      acc[i] = r == 0 ? part[i] : op == 0 ? acc[i] + part[i] : op == 1 ? std::min(acc[i], part[i]) : std::max(acc[i], part[i]);
+  }
+  for (int r = 0; r < n; ++r) {
+    CUDA_TRY(cudaMemcpyAsync(buf[r], acc.data(), count * sizeof(double), cudaMemcpyHostToDevice, hs[r]->stream));
+    CUDA_TRY(cudaStreamSynchronize(hs[r]->stream));
+  }
+  return BLAST_CF_OK;
+}
+
+int owner_weights(const blast_cf *h, double *out) {
+  std::fill(out, out + h->nn, 1.0);
+  if (!h->xch) return BLAST_CF_OK;
+  const Exchange *x = h->xch;
+  for (int i = 0; i < x->num_nbr; ++i)   // a neighbour with a lower rank owns every node it shares with us
+    if (x->nbr_rank[i] < x->rank)
+      for (int64_t r = x->nbr_offset[i]; r < x->nbr_offset[i + 1]; ++r) out[x->h_rows[r]] = 0.0;
+  return BLAST_CF_OK;
+}
 
 }  // namespace blastcf
 

@@ -145,6 +145,7 @@ struct Exchange {
   int64_t nn = 0, nrows = 0, nu = 0;
   std::vector<int32_t> nbr_rank;
   std::vector<int64_t> nbr_offset;
+  std::vector<int32_t> h_rows;   // host copy of the shared-node rows (nbr_nodes)
   cudaStream_t stream = nullptr;
   int32_t *d_rows = nullptr, *d_unodes = nullptr;
   int64_t *d_sptr = nullptr, *d_src = nullptr;

@@ -38,21 +38,22 @@ struct V5Dims {
   static constexpr int OFF_J = OFF_W + WREG;            // J0^{-1} + gamma for the two buffers [2][10]
   static constexpr int OFF_RED = OFF_J + 20;
   static constexpr int OFF_ID = OFF_RED + 32;          // zone -> node ids of the next two zones, int32 [2][P^3]
-  static constexpr int TOTAL = OFF_ID + (2 * P3 + 1) / 2;
+  static constexpr int OFF_MB = OFF_ID + (2 * P3 + 1) / 2;   // two mbarriers (kb1_v10.cuh bulk copies)
+  static constexpr int TOTAL = OFF_MB + 2;
   static constexpr int MT = (N + 7) / 8, KS_P = (P + 3) / 4, KS_N = (N + 3) / 4, KS_T = (T + 3) / 4;
 };
 
 // MODE picks the register split between the point warps and the DMMA warps (setmaxnreg) and the DMMA
-// tiles in flight per warp: 0 = 168 / 88 / 8, 1 = 184 / 72 / 4, 2 = 200 / 56 / 2.
+// tiles in flight per warp: 0 = 168 / 88 / 8, 1 = 184 / 72 / 4, 2 = 200 / 56 / 2, 3 = 176 / 80 / 4.
 template <int K, int MODE = 0>
 struct KB1V5Cfg {
   using Dm = V5Dims<K>;
   static constexpr int NPW = (Dm::N3 / 2 + 127) / 128 * 128;   // 2 points per point-thread
   static constexpr int NKW = 256;
   static constexpr int NTH = NPW + NKW;
-  static constexpr int REG_PW = MODE == 0 ? 168 : MODE == 1 ? 184 : 200;
-  static constexpr int REG_KW = MODE == 0 ? 88 : MODE == 1 ? 72 : 56;
-  static constexpr int KWCH = MODE == 0 ? 8 : MODE == 1 ? 4 : 2;   // DMMA tiles in flight per warp
+  static constexpr int REG_PW = MODE == 0 ? 168 : MODE == 1 ? 184 : MODE == 2 ? 200 : 176;
+  static constexpr int REG_KW = MODE == 0 ? 88 : MODE == 1 ? 72 : MODE == 2 ? 56 : 80;
+  static constexpr int KWCH = MODE == 0 ? 8 : MODE == 1 ? 4 : MODE == 2 ? 2 : 4;   // DMMA tiles in flight per warp
   static constexpr int REG_LAUNCH = (65536 / NTH) / 8 * 8;
   static_assert(NPW * REG_PW + NKW * REG_KW <= NTH * REG_LAUNCH, "register split exceeds the CTA's allocation");
   static constexpr int SMEM_BYTES = Dm::TOTAL * 8;
