@@ -183,6 +183,13 @@ int blast_cf_exchange_plan(int32_t rank, int32_t num_neighbors, const int32_t *n
                            int64_t *src_ptr, int64_t *src);
 
 /* Size of ncclUniqueId (bytes) and a helper so Python can create it without linking NCCL itself. */
+/* Host-only (no CUDA): the owner weights of a rank's local nodes used by the multi-rank integrator's dot
+ * products — out[n] = 0 if a neighbour with a lower rank shares node n, else 1 (each shared node is
+ * counted by its lowest-ranked holder; MFEM's group masters).  Arguments as in
+ * blast_cf_mesh; out: HOST [num_nodes].  EINVAL for NULL arguments or node ids out of range. */
+int blast_cf_owner_mask(int32_t rank, int32_t num_neighbors, const int32_t *nbr_rank, const int64_t *nbr_offset,
+                        const int32_t *nbr_nodes, int64_t num_nodes, double *out);
+
 int blast_cf_nccl_unique_id_size(void);
 int blast_cf_nccl_get_unique_id(void *out);
 
@@ -205,7 +212,12 @@ int blast_cf_nccl_get_unique_id(void *out);
  *   - time stepping: the RK2-average scheme (reading R22), which conserves the discrete total
  *     energy 1/2 v^T M_V v + sum_z 1^T M_E e_z up to the CG tolerance (the paper's Table 6 check,
  *     PAPER.md:894-900); reflecting walls v.n = 0 on the bounding box of x0 (reading R23).
- * Single GPU (mesh->nranks == 1) in this version.
+ * Multi-GPU: with a multi-rank corner-force handle every call below is collective over
+ * the ranks (each process calls it for its rank; NCCL inside).  The CG for M_V adds the shared-node sum
+ * of A p to every iteration (the ascending-rank exchange of blast_cf_eval) and sums its dot products over
+ * the ranks with each shared node counted by its lowest-ranked holder, so all ranks keep identical
+ * scalars and, on shared nodes, bitwise identical iterates; the energies are group totals.  Loopback
+ * groups (n ranks on one device, tests) are driven by the *_loopback entries below.
  * --------------------------------------------------------------------------------------------- */
 typedef struct blast_cf_rk2 blast_cf_rk2; /* opaque; borrows the corner-force handle h (same stream) */
 
@@ -213,15 +225,18 @@ typedef struct {
   double cg_rel_tol;      /* 1e-14: per component, stop when ||r|| <= tol * ||b|| (residual 2-norm) */
   int32_t cg_max_iter;    /* 500 */
   int32_t cg_check_every; /* 8: iterations between host-side convergence checks */
-  int32_t wall_bc;        /* 1: v . n = 0 on the walls of the bounding box of x0; 0: free */
+  int32_t wall_bc;        /* 1: v . n = 0 on the walls of the global box; 0: free */
+  double box_lo[3], box_hi[3]; /* the global box of the walls; used when box_hi[0] > box_lo[0], else derived:
+                                  the bounding box of x0 (one rank) or its min / max over the NCCL ranks
+                                  (a collective inside create); loopback groups must give it */
 } blast_cf_rk2_opts;
 
 void blast_cf_rk2_default_opts(blast_cf_rk2_opts *o);
 
 /* Create the integrator for handle h.  mesh: the mesh h was created from (HOST pointers; x0 gives the
  * walls).  rho0detJ0: HOST [num_zones][Nq], copied (the integrator evaluates the force with this copy).
- * Allocates all device workspace.  BLAST_CF_EUNSUPPORTED for nranks > 1, or for dense M_E^{-1} zones
- * beyond 2^34 long-double flops at create. */
+ * Allocates all device workspace.  Multi-rank NCCL handles: collective (walls, Jacobi diagonal).
+ * BLAST_CF_EUNSUPPORTED for dense M_E^{-1} zones beyond 2^34 long-double flops at create. */
 int blast_cf_rk2_create(blast_cf *h, const blast_cf_mesh *mesh, const double *rho0detJ0,
                         const blast_cf_rk2_opts *opts, blast_cf_rk2 **out);
 
@@ -256,6 +271,18 @@ int blast_cf_rk2_mass_apply(blast_cf_rk2 *s, const double *u, double *out);
 /* Discrete energies (HOST outputs): kinetic = 1/2 sum_c v_c^T M_V v_c, internal = sum_z 1^T M_E e_z.
  * v, e DEVICE.  Deterministic.  Synchronous. */
 int blast_cf_rk2_energy(blast_cf_rk2 *s, const double *v, const double *e, double *kinetic, double *internal);
+
+/* Tests on one device (multi-GPU logic without NCCL): S[r] is the integrator of rank r of an n-rank
+ * loopback group (corner-force handles created with nranks = n and no NCCL id, opts->box_lo/box_hi set).
+ * setup_loopback completes their creation (shared-node sum of the Jacobi diagonal; call once, after all
+ * n creates).  rates_loopback / energy_loopback are blast_cf_rk2_rates / blast_cf_rk2_energy of the whole
+ * group: per-rank DEVICE arrays, out_dt / cg_iters / kinetic / internal HOST (group values).  Synchronous. */
+int blast_cf_rk2_setup_loopback(blast_cf_rk2 *const *S, int n);
+int blast_cf_rk2_rates_loopback(blast_cf_rk2 *const *S, int n, const double *const *x, const double *const *v,
+                                const double *const *e, const double *const *vbar, double *const *out_dvdt,
+                                double *const *out_dedt, double *out_dt, int32_t *cg_iters);
+int blast_cf_rk2_energy_loopback(blast_cf_rk2 *const *S, int n, const double *const *v, const double *const *e,
+                                 double *kinetic, double *internal);
 
 int blast_cf_rk2_destroy(blast_cf_rk2 *s);
 

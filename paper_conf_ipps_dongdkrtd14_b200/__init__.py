@@ -50,7 +50,7 @@ class Params(ctypes.Structure):
 
 class RK2Opts(ctypes.Structure):
     _fields_ = [("cg_rel_tol", ctypes.c_double), ("cg_max_iter", ctypes.c_int32), ("cg_check_every", ctypes.c_int32),
-                ("wall_bc", ctypes.c_int32)]
+                ("wall_bc", ctypes.c_int32), ("box_lo", ctypes.c_double * 3), ("box_hi", ctypes.c_double * 3)]
 
 
 class Info(ctypes.Structure):
@@ -97,6 +97,7 @@ def lib():
     L.blast_cf_nccl_unique_id_size.argtypes = []
     L.blast_cf_nccl_get_unique_id.argtypes = [vp]
     L.blast_cf_exchange_plan.argtypes = [i32, i32, vp, vp, vp, i64, ctypes.POINTER(i64), vp, vp, vp]
+    L.blast_cf_owner_mask.argtypes = [i32, i32, vp, vp, vp, i64, vp]
     L.blast_cf_debug_cta_dt.argtypes = [vp, vp, i64, ctypes.POINTER(i32), ctypes.POINTER(i32)]
     L.blast_cf_debug_stage_clocks.argtypes = [vp, vp, i64]
     L.blast_cf_eval_loopback.argtypes = [vp, ctypes.c_int, vp, vp, vp, vp, vp, vp, vp]
@@ -113,11 +114,17 @@ def lib():
                                        ctypes.POINTER(ctypes.c_double), ctypes.POINTER(i32), ctypes.POINTER(i32)]
     L.blast_cf_rk2_energy.argtypes = [vp, vp, vp, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]
     L.blast_cf_rk2_destroy.argtypes = [vp]
+    L.blast_cf_rk2_setup_loopback.argtypes = [vp, ctypes.c_int]
+    L.blast_cf_rk2_rates_loopback.argtypes = [vp, ctypes.c_int] + [vp] * 6 + [ctypes.POINTER(ctypes.c_double),
+                                                                             ctypes.POINTER(i32)]
+    L.blast_cf_rk2_energy_loopback.argtypes = [vp, ctypes.c_int, vp, vp, ctypes.POINTER(ctypes.c_double),
+                                               ctypes.POINTER(ctypes.c_double)]
     for f in ("blast_cf_rk2_create", "blast_cf_rk2_step", "blast_cf_rk2_rates", "blast_cf_rk2_mass_apply",
-              "blast_cf_rk2_energy", "blast_cf_rk2_destroy", "blast_cf_rk2_advance",
+              "blast_cf_rk2_energy", "blast_cf_rk2_destroy", "blast_cf_rk2_advance", "blast_cf_rk2_setup_loopback",
+              "blast_cf_rk2_rates_loopback", "blast_cf_rk2_energy_loopback",
               "blast_cf_create", "blast_cf_eval", "blast_cf_eval_host", "blast_cf_eval_debug_Fz", "blast_cf_get_info",
               "blast_cf_set_timing", "blast_cf_kernel_times", "blast_cf_destroy", "blast_cf_nccl_unique_id_size",
-              "blast_cf_nccl_get_unique_id", "blast_cf_exchange_plan", "blast_cf_debug_cta_dt",
+              "blast_cf_nccl_get_unique_id", "blast_cf_exchange_plan", "blast_cf_owner_mask", "blast_cf_debug_cta_dt",
               "blast_cf_debug_stage_clocks", "blast_cf_eval_loopback", "blast_cf_autotune"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
@@ -157,6 +164,17 @@ def exchange_plan(rank: int, nbr_rank: np.ndarray, nbr_offset: np.ndarray, nbr_n
                                         sptr.ctypes.data, src.ctypes.data), "blast_cf_exchange_plan")
     n = nu.value
     return uniq[:n].copy(), sptr[:n + 1].copy(), src[:sptr[n]].copy()
+
+
+def owner_mask(rank: int, nbr_rank: np.ndarray, nbr_offset: np.ndarray, nbr_nodes: np.ndarray, num_nodes: int):
+    """The library's owner weights of a rank's local nodes (host only; see blast_cf_owner_mask)."""
+    nbr_rank = np.ascontiguousarray(nbr_rank, dtype=np.int32)
+    nbr_offset = np.ascontiguousarray(nbr_offset, dtype=np.int64)
+    nbr_nodes = np.ascontiguousarray(nbr_nodes, dtype=np.int32)
+    out = np.zeros(max(int(num_nodes), 1))
+    _check(lib().blast_cf_owner_mask(rank, len(nbr_rank), _ptr(nbr_rank, np.int32), _ptr(nbr_offset, np.int64),
+                                     _ptr(nbr_nodes, np.int32), int(num_nodes), out.ctypes.data), "blast_cf_owner_mask")
+    return out[:int(num_nodes)]
 
 
 class CornerForce:
@@ -429,6 +447,38 @@ def eval_loopback(handles, xs, vs, es, rs):
     _check(lib().blast_cf_eval_loopback(hs, n, arr(xs), arr(vs), arr(es), arr(rs), arr([o[0] for o in outs]),
                                         arr([o[1] for o in outs]), arr([o[2] for o in outs])), "blast_cf_eval_loopback")
     return outs
+
+
+def rk2_setup_loopback(rk2s):
+    """Complete the creation of a loopback group's integrators (blast_cf_rk2_setup_loopback)."""
+    P = ctypes.c_void_p * len(rk2s)
+    _check(lib().blast_cf_rk2_setup_loopback(P(*[r._h for r in rk2s]), len(rk2s)), "blast_cf_rk2_setup_loopback")
+
+
+def rk2_rates_loopback(rk2s, xs, vs, es, vbars=None):
+    """RK2.rates of a whole loopback group (one GPU): per-rank (dv/dt, de/dt) tensors, group dt, CG iterations."""
+    import torch
+    n = len(rk2s)
+    P = ctypes.c_void_p * n
+    arr = lambda ts: P(*[None if t is None else ctypes.c_void_p(t.data_ptr()) for t in ts])
+    dvs = [torch.empty((r.cf.dim, r.cf.num_nodes), dtype=torch.float64, device=r.cf.device) for r in rk2s]
+    des = [torch.empty((r.cf.num_zones, r.cf.nt), dtype=torch.float64, device=r.cf.device) for r in rk2s]
+    d, it = ctypes.c_double(0.0), ctypes.c_int32(0)
+    _check(lib().blast_cf_rk2_rates_loopback(P(*[r._h for r in rk2s]), n, arr(xs), arr(vs), arr(es),
+                                             arr(vbars if vbars is not None else [None] * n), arr(dvs), arr(des),
+                                             ctypes.byref(d), ctypes.byref(it)), "blast_cf_rk2_rates_loopback")
+    return dvs, des, d.value, it.value
+
+
+def rk2_energy_loopback(rk2s, vs, es):
+    """(kinetic, internal) energies of a whole loopback group."""
+    n = len(rk2s)
+    P = ctypes.c_void_p * n
+    arr = lambda ts: P(*[ctypes.c_void_p(t.data_ptr()) for t in ts])
+    ke, ie = ctypes.c_double(0.0), ctypes.c_double(0.0)
+    _check(lib().blast_cf_rk2_energy_loopback(P(*[r._h for r in rk2s]), n, arr(vs), arr(es), ctypes.byref(ke),
+                                              ctypes.byref(ie)), "blast_cf_rk2_energy_loopback")
+    return ke.value, ie.value
 
 
 def nccl_unique_id() -> bytes:

@@ -810,13 +810,12 @@ int group_allreduce(blast_cf *const *hs, int n, double *const *buf, int count, i
 }
 
 int owner_weights(const blast_cf *h, double *out) {
-  std::fill(out, out + h->nn, 1.0);
-  if (!h->xch) return BLAST_CF_OK;
-  const Exchange *x = h->xch;
-  for (int i = 0; i < x->num_nbr; ++i)   // a neighbour with a lower rank owns every node it shares with us
-    if (x->nbr_rank[i] < x->rank)
-      for (int64_t r = x->nbr_offset[i]; r < x->nbr_offset[i + 1]; ++r) out[x->h_rows[r]] = 0.0;
-  return BLAST_CF_OK;
+  if (!h->xch) {
+    std::fill(out, out + h->nn, 1.0);
+    return BLAST_CF_OK;
+  }
+  const Exchange *x = h->xch;   // a neighbour with a lower rank owns every node it shares with us
+  return blast_cf_owner_mask(x->rank, x->num_nbr, x->nbr_rank.data(), x->nbr_offset.data(), x->h_rows.data(), h->nn, out);
 }
 
 }  // namespace blastcf
@@ -1141,6 +1140,21 @@ int blast_cf_exchange_plan(int32_t rank, int32_t num_neighbors, const int32_t *n
   std::copy(pl.unique_nodes.begin(), pl.unique_nodes.end(), unique_nodes);
   std::copy(pl.src_ptr.begin(), pl.src_ptr.end(), src_ptr);
   std::copy(pl.src.begin(), pl.src.end(), src);
+  return BLAST_CF_OK;
+}
+
+int blast_cf_owner_mask(int32_t rank, int32_t num_neighbors, const int32_t *nbr_rank, const int64_t *nbr_offset,
+                        const int32_t *nbr_nodes, int64_t num_nodes, double *out) {
+  if (num_neighbors < 0 || num_nodes < 0 || (num_nodes > 0 && !out) ||
+      (num_neighbors > 0 && (!nbr_rank || !nbr_offset || !nbr_nodes)))
+    return fail(BLAST_CF_EINVAL, "NULL argument");
+  std::fill(out, out + num_nodes, 1.0);
+  for (int i = 0; i < num_neighbors; ++i)   // the same rule as the integrator's owner weights
+    if (nbr_rank[i] < rank)
+      for (int64_t r = nbr_offset[i]; r < nbr_offset[i + 1]; ++r) {
+        if (nbr_nodes[r] < 0 || nbr_nodes[r] >= num_nodes) return fail(BLAST_CF_EINVAL, "nbr_nodes[%lld]", (long long)r);
+        out[nbr_nodes[r]] = 0.0;
+      }
   return BLAST_CF_OK;
 }
 

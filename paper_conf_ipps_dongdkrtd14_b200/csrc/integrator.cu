@@ -378,10 +378,11 @@ __global__ void __launch_bounds__(NB) k_gather(NodeArgs na, const double *__rest
 }
 
 // CG start: X = 0, R = mask (sgn b), Z = R / diag, P = 0; rz, bb
-template <int D>
+template <int D, bool MULTI = false>
 __global__ void __launch_bounds__(NB) k_cg_init(NodeArgs na, double sgn, const double *__restrict__ b,
                                                 const double *__restrict__ invd, double *X, double *R, double *Zv,
-                                                double *P, double *partials, CGScal *sc) {
+                                                double *P, double *partials, CGScal *sc,
+                                                const double *__restrict__ own = nullptr, double *red = nullptr) {
   const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   double v[2 * D];
 #pragma unroll
@@ -394,10 +395,16 @@ __global__ void __launch_bounds__(NB) k_cg_init(NodeArgs na, double sgn, const d
       zz = r * id;
       X[g] = 0.0; R[g] = r; Zv[g] = zz; P[g] = 0.0;
     }
-    v[c] = r * zz;
-    v[D + c] = r * r;
+    const double w = (MULTI && n < na.nn) ? own[n] : 1.0;   // each shared node counted by its owner only
+    v[c] = w * r * zz;
+    v[D + c] = w * r * r;
   }
   if (grid_sum<2 * D>(v, partials, &sc->ticket) && threadIdx.x == 0) {
+    if (MULTI) {   // local sums; k_cg_scal finishes after the group allreduce
+#pragma unroll
+      for (int c = 0; c < 2 * D; ++c) red[c] = v[c];
+      return;
+    }
     bool done = true;
     for (int c = 0; c < D; ++c) {
       sc->rz[c] = v[c]; sc->bb[c] = v[D + c]; sc->rr[c] = v[D + c]; sc->beta[c] = 0.0; sc->alpha[c] = 0.0;
@@ -409,7 +416,7 @@ __global__ void __launch_bounds__(NB) k_cg_init(NodeArgs na, double sgn, const d
 }
 
 // AP = mask (sum of zone actions), P = Z + beta P; alpha = rz / (P . AP)
-template <int D>
+template <int D, bool DOT = true>
 __global__ void __launch_bounds__(NB) k_cg_gather(NodeArgs na, const double *__restrict__ Y,
                                                   const double *__restrict__ invd, const double *__restrict__ Zv,
                                                   double *P, double *AP, double *partials, CGScal *sc) {
@@ -431,15 +438,60 @@ __global__ void __launch_bounds__(NB) k_cg_gather(NodeArgs na, const double *__r
       v[c] = pn * ap;
     }
   }
+  if (!DOT) return;   // multi-rank: AP still needs its shared-node sum before P . AP (k_cg_pap)
   if (grid_sum<D>(v, partials, &sc->ticket) && threadIdx.x == 0)
     for (int c = 0; c < D; ++c) sc->alpha[c] = v[c] > 0.0 ? sc->rz[c] / v[c] : 0.0;
 }
 
-// X += alpha P, R -= alpha AP, Z = R / diag; beta = rz' / rz; convergence
+// multi-rank: owned P . AP (after the shared-node sum of AP) -> red[0, D)
 template <int D>
+__global__ void __launch_bounds__(NB) k_cg_pap(int64_t nn, const double *__restrict__ P, const double *__restrict__ AP,
+                                               const double *__restrict__ own, double *partials, CGScal *sc,
+                                               double *red) {
+  if (sc->done) return;
+  const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  double v[D];
+#pragma unroll
+  for (int c = 0; c < D; ++c) v[c] = n < nn ? own[n] * P[c * nn + n] * AP[c * nn + n] : 0.0;
+  if (grid_sum<D>(v, partials, &sc->ticket) && threadIdx.x == 0)
+#pragma unroll
+    for (int c = 0; c < D; ++c) red[c] = v[c];
+}
+
+// multi-rank scalar steps on the group-reduced sums (one thread):
+//   PH 0 (after init): rz, bb, rr from red[0, 2D);  PH 1: alpha from red[0, D);  PH 2: beta, rr, done
+template <int D, int PH>
+__global__ void k_cg_scal(const double *__restrict__ red, CGScal *sc) {
+  if (PH != 0 && sc->done) return;
+  if (PH == 0) {
+    bool done = true;
+    for (int c = 0; c < D; ++c) {
+      sc->rz[c] = red[c]; sc->bb[c] = red[D + c]; sc->rr[c] = red[D + c]; sc->beta[c] = 0.0; sc->alpha[c] = 0.0;
+      done = done && red[D + c] == 0.0;
+    }
+    sc->done = done ? 1 : 0;
+    sc->iters = 0;
+  } else if (PH == 1) {
+    for (int c = 0; c < D; ++c) sc->alpha[c] = red[c] > 0.0 ? sc->rz[c] / red[c] : 0.0;
+  } else {
+    bool done = true;
+    for (int c = 0; c < D; ++c) {
+      sc->beta[c] = sc->rz[c] > 0.0 ? red[c] / sc->rz[c] : 0.0;
+      sc->rz[c] = red[c];
+      sc->rr[c] = red[D + c];
+      done = done && red[D + c] <= sc->tol2 * sc->bb[c];
+    }
+    sc->iters += 1;
+    sc->done = done ? 1 : 0;
+  }
+}
+
+// X += alpha P, R -= alpha AP, Z = R / diag; beta = rz' / rz; convergence
+template <int D, bool MULTI = false>
 __global__ void __launch_bounds__(NB) k_cg_update(NodeArgs na, const double *__restrict__ invd, double *X, double *R,
                                                   double *Zv, const double *__restrict__ P,
-                                                  const double *__restrict__ AP, double *partials, CGScal *sc) {
+                                                  const double *__restrict__ AP, double *partials, CGScal *sc,
+                                                  const double *__restrict__ own = nullptr, double *red = nullptr) {
   if (sc->done) return;
   const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   double v[2 * D];
@@ -454,10 +506,16 @@ __global__ void __launch_bounds__(NB) k_cg_update(NodeArgs na, const double *__r
       zz = r * invd[g];
       R[g] = r; Zv[g] = zz;
     }
-    v[c] = r * zz;
-    v[D + c] = r * r;
+    const double w = (MULTI && n < na.nn) ? own[n] : 1.0;
+    v[c] = w * r * zz;
+    v[D + c] = w * r * r;
   }
   if (grid_sum<2 * D>(v, partials, &sc->ticket) && threadIdx.x == 0) {
+    if (MULTI) {
+#pragma unroll
+      for (int c = 0; c < 2 * D; ++c) red[c] = v[c];
+      return;
+    }
     bool done = true;
     for (int c = 0; c < D; ++c) {
       sc->beta[c] = sc->rz[c] > 0.0 ? v[c] / sc->rz[c] : 0.0;
@@ -481,7 +539,7 @@ __global__ void __launch_bounds__(NB) k_axpy(double *out, const double *a, doubl
 template <int D>
 __global__ void __launch_bounds__(NB) k_gather_dot(NodeArgs na, const double *__restrict__ Y,
                                                    const double *__restrict__ u, double *partials, unsigned *ticket,
-                                                   double *out) {
+                                                   double *out, const double *__restrict__ own = nullptr) {
   const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   double v[1] = {0.0};
   if (n < na.nn) {
@@ -489,6 +547,22 @@ __global__ void __launch_bounds__(NB) k_gather_dot(NodeArgs na, const double *__
     gather_node<D>(na, Y, n, s);
 #pragma unroll
     for (int c = 0; c < D; ++c) v[0] += u[c * na.nn + n] * s[c];
+    if (own) v[0] *= own[n];
+  }
+  if (grid_sum<1>(v, partials, ticket) && threadIdx.x == 0) *out = v[0];
+}
+
+// owner-weighted sum_c a_c . b_c over the local nodes ([dim][nn] vectors) -> *out
+template <int D>
+__global__ void __launch_bounds__(NB) k_wdot(int64_t nn, const double *__restrict__ a, const double *__restrict__ b,
+                                             const double *__restrict__ own, double *partials, unsigned *ticket,
+                                             double *out) {
+  const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  double v[1] = {0.0};
+  if (n < nn) {
+#pragma unroll
+    for (int c = 0; c < D; ++c) v[0] += a[c * nn + n] * b[c * nn + n];
+    v[0] *= own[n];
   }
   if (grid_sum<1>(v, partials, ticket) && threadIdx.x == 0) *out = v[0];
 }
@@ -521,6 +595,10 @@ struct blast_cf_rk2 {
   double *scal_out = nullptr;   // [4] energies / dots
   unsigned *ticket = nullptr;
   CGScal *sc = nullptr;
+  // multi-rank: owner weights of the local nodes, group-reduction buffer
+  bool multi = false, loopback = false, ready = false;
+  double *own = nullptr, *red = nullptr;
+  std::vector<unsigned char> fixed;   // [dim][nn] wall DOFs (host; the Jacobi diagonal is inverted after its shared-node sum)
   // host
   CGScal *h_sc = nullptr;   // pinned
   size_t smem_mass = 0, smem_diag = 0, smem_me1 = 0, smem_rhs = 0;
@@ -532,7 +610,7 @@ void free_rk2(blast_cf_rk2 *s) {
   if (!s) return;
   double *bufs[] = {s->R, s->Sq, s->F1, s->FTv, s->dtd, s->DV, s->Vb, s->DE, s->xh, s->eh, s->Rr, s->Zv, s->P,
                     s->AP, s->Y, s->invd, s->partials, s->me1, s->m1inv, s->zscale, s->Minv, s->scal_out,
-                    s->bx, s->bv, s->be};
+                    s->bx, s->bv, s->be, s->own, s->red};
   for (double *b : bufs) cudaFree(b);
   cudaFree(s->ticket);
   cudaFree(s->sc);
@@ -563,6 +641,79 @@ void launch_mass_zone(blast_cf_rk2 *s, const double *u, const double *Pold, cons
 int check(const char *what) {
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(BLAST_CF_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+  return BLAST_CF_OK;
+}
+
+int cg_solve(blast_cf_rk2 *s, const double *b, double sgn, double *X, int *iters_out);
+
+// Multi-rank CG (f2): the group's ranks (n = 1 under NCCL, all n of a loopback group) run the same
+// Jacobi PCG as cg_solve in lockstep; each iteration adds the shared-node sum of A p (the M_V action of a
+// partition misses its neighbours' zones) and group sums of the owner-weighted dot products, so every
+// rank holds the same scalars and, on shared nodes, bitwise the same iterates.
+int cg_group(blast_cf_rk2 *const *S, int n, const double *const *b, double sgn, double *const *X, int *iters_out) {
+  if (n == 1 && !S[0]->multi) return cg_solve(S[0], b[0], sgn, X[0], iters_out);
+  std::vector<blast_cf *> hs(n);
+  std::vector<double *> red(n), ap(n);
+  for (int r = 0; r < n; ++r) { hs[r] = S[r]->h; red[r] = S[r]->red; ap[r] = S[r]->AP; }
+  const int D = S[0]->hv.dim;
+  int rc;
+  for (int r = 0; r < n; ++r) {
+    blast_cf_rk2 *s = S[r];
+    const NodeArgs na = node_args(s);
+    const unsigned nb = blocks_for(s->hv.nn, NB);
+    if (D == 3) k_cg_init<3, true><<<nb, NB, 0, s->hv.stream>>>(na, sgn, b[r], s->invd, X[r], s->Rr, s->Zv, s->P, s->partials, s->sc, s->own, s->red);
+    else k_cg_init<2, true><<<nb, NB, 0, s->hv.stream>>>(na, sgn, b[r], s->invd, X[r], s->Rr, s->Zv, s->P, s->partials, s->sc, s->own, s->red);
+  }
+  if ((rc = blastcf::group_allreduce(hs.data(), n, red.data(), 2 * D, 0))) return rc;
+  for (int r = 0; r < n; ++r) {
+    if (D == 3) k_cg_scal<3, 0><<<1, 1, 0, S[r]->hv.stream>>>(S[r]->red, S[r]->sc);
+    else k_cg_scal<2, 0><<<1, 1, 0, S[r]->hv.stream>>>(S[r]->red, S[r]->sc);
+  }
+  int it = 0;
+  const int every = std::max(1, S[0]->opts.cg_check_every);
+  while (true) {
+    CUDA_TRY(cudaMemcpyAsync(S[0]->h_sc, S[0]->sc, sizeof(CGScal), cudaMemcpyDeviceToHost, S[0]->hv.stream));
+    CUDA_TRY(cudaStreamSynchronize(S[0]->hv.stream));
+    if (S[0]->h_sc->done || it >= S[0]->opts.cg_max_iter) break;
+    for (int j = 0; j < every && it < S[0]->opts.cg_max_iter; ++j, ++it) {
+      for (int r = 0; r < n; ++r) {   // A p on every partition (p = z + beta p formed inside)
+        blast_cf_rk2 *s = S[r];
+        const unsigned nb = blocks_for(s->hv.nn, NB);
+        launch_mass_zone(s, s->Zv, s->P, s->sc);
+        if (D == 3) k_cg_gather<3, false><<<nb, NB, 0, s->hv.stream>>>(node_args(s), s->Y, s->invd, s->Zv, s->P, s->AP, s->partials, s->sc);
+        else k_cg_gather<2, false><<<nb, NB, 0, s->hv.stream>>>(node_args(s), s->Y, s->invd, s->Zv, s->P, s->AP, s->partials, s->sc);
+      }
+      if ((rc = blastcf::group_exchange_sum(hs.data(), n, ap.data()))) return rc;
+      for (int r = 0; r < n; ++r) {
+        blast_cf_rk2 *s = S[r];
+        const unsigned nb = blocks_for(s->hv.nn, NB);
+        if (D == 3) k_cg_pap<3><<<nb, NB, 0, s->hv.stream>>>(s->hv.nn, s->P, s->AP, s->own, s->partials, s->sc, s->red);
+        else k_cg_pap<2><<<nb, NB, 0, s->hv.stream>>>(s->hv.nn, s->P, s->AP, s->own, s->partials, s->sc, s->red);
+      }
+      if ((rc = blastcf::group_allreduce(hs.data(), n, red.data(), D, 0))) return rc;
+      for (int r = 0; r < n; ++r) {
+        blast_cf_rk2 *s = S[r];
+        const unsigned nb = blocks_for(s->hv.nn, NB);
+        if (D == 3) {
+          k_cg_scal<3, 1><<<1, 1, 0, s->hv.stream>>>(s->red, s->sc);
+          k_cg_update<3, true><<<nb, NB, 0, s->hv.stream>>>(node_args(s), s->invd, X[r], s->Rr, s->Zv, s->P, s->AP, s->partials, s->sc, s->own, s->red);
+        } else {
+          k_cg_scal<2, 1><<<1, 1, 0, s->hv.stream>>>(s->red, s->sc);
+          k_cg_update<2, true><<<nb, NB, 0, s->hv.stream>>>(node_args(s), s->invd, X[r], s->Rr, s->Zv, s->P, s->AP, s->partials, s->sc, s->own, s->red);
+        }
+      }
+      if ((rc = blastcf::group_allreduce(hs.data(), n, red.data(), 2 * D, 0))) return rc;
+      for (int r = 0; r < n; ++r) {
+        if (D == 3) k_cg_scal<3, 2><<<1, 1, 0, S[r]->hv.stream>>>(S[r]->red, S[r]->sc);
+        else k_cg_scal<2, 2><<<1, 1, 0, S[r]->hv.stream>>>(S[r]->red, S[r]->sc);
+      }
+    }
+    if ((rc = check("group CG kernels"))) return rc;
+  }
+  if (iters_out) *iters_out = S[0]->h_sc->iters;
+  if (!S[0]->h_sc->done)
+    return fail(BLAST_CF_EUNSUPPORTED, "CG did not converge in %d iterations (rel tol %g)", S[0]->opts.cg_max_iter,
+                S[0]->opts.cg_rel_tol);
   return BLAST_CF_OK;
 }
 
@@ -647,6 +798,103 @@ bool invert_ld(std::vector<long double> &a, int m) {
   return true;
 }
 
+// shared-node sum of the gathered mass diagonal over the group, then invd = 1/diag (0 on wall DOFs)
+int finish_setup(blast_cf_rk2 *const *S, int n) {
+  int rc;
+  if (S[0]->multi) {
+    std::vector<blast_cf *> hs(n);
+    std::vector<double *> v(n);
+    for (int r = 0; r < n; ++r) { hs[r] = S[r]->h; v[r] = S[r]->invd; }
+    if ((rc = blastcf::group_exchange_sum(hs.data(), n, v.data()))) return rc;
+  }
+  for (int r = 0; r < n; ++r) {
+    blast_cf_rk2 *s = S[r];
+    const int64_t nx = s->nx;
+    std::vector<double> diag(std::max<int64_t>(nx, 1), 0.0);
+    if (nx > 0) CUDA_TRY(cudaMemcpyAsync(diag.data(), s->invd, nx * sizeof(double), cudaMemcpyDeviceToHost, s->hv.stream));
+    CUDA_TRY(cudaStreamSynchronize(s->hv.stream));
+    for (int64_t i = 0; i < nx; ++i) {
+      double &d = diag[i];
+      if (!(d > 0.0) && !s->fixed[i])
+        return fail(BLAST_CF_EINVAL, "non-positive mass diagonal at DOF %lld of rank %d", (long long)i, r);
+      d = s->fixed[i] ? 0.0 : 1.0 / d;
+    }
+    if (nx > 0) CUDA_TRY(cudaMemcpy(s->invd, diag.data(), nx * sizeof(double), cudaMemcpyHostToDevice));
+    s->ready = true;
+  }
+  return BLAST_CF_OK;
+}
+
+// dv/dt = -M_V^{-1} F.1 and de/dt = M_E^{-1} F^T vbar on every rank of the group
+int rates_group(blast_cf_rk2 *const *S, int n, const double *const *x, const double *const *v, const double *const *e,
+                const double *const *vbar, double *const *out_dvdt, double *const *out_dedt, double *out_dt,
+                int32_t *cg_iters) {
+  int rc;
+  std::vector<blast_cf *> hs(n);
+  std::vector<double *> f1(n), dtd(n);
+  for (int r = 0; r < n; ++r) {
+    blast_cf_rk2 *s = S[r];
+    hs[r] = s->h; f1[r] = s->F1; dtd[r] = s->dtd;
+    if ((rc = blastcf::eval_with_S(s->h, x[r], v[r], e[r], s->R, s->F1, s->FTv, s->dtd, s->Sq))) return rc;
+  }
+  if (S[0]->loopback) {   // (an NCCL rank's evaluation already summed F.1 and reduced dt)
+    if ((rc = blastcf::group_exchange_sum(hs.data(), n, f1.data()))) return rc;
+    if ((rc = blastcf::group_allreduce(hs.data(), n, dtd.data(), 1, 1))) return rc;
+  }
+  int it = 0;
+  if ((rc = cg_group(S, n, f1.data(), -1.0, out_dvdt, &it))) return rc;
+  if (cg_iters) *cg_iters = it;
+  for (int r = 0; r < n; ++r) launch_energy_rhs(S[r], vbar && vbar[r] ? vbar[r] : v[r], out_dedt[r]);
+  if ((rc = check("energy rhs"))) return rc;
+  if (out_dt) CUDA_TRY(cudaMemcpyAsync(out_dt, S[0]->dtd, sizeof(double), cudaMemcpyDeviceToHost, S[0]->hv.stream));
+  for (int r = 0; r < n; ++r) CUDA_TRY(cudaStreamSynchronize(S[r]->hv.stream));
+  return BLAST_CF_OK;
+}
+
+// kinetic = 1/2 sum_c v_c^T M_V v_c and internal = sum_z 1^T M_E e_z over the whole group (shared nodes:
+// (M_V v) summed over their sharers, then counted by the owner)
+int energy_group(blast_cf_rk2 *const *S, int n, const double *const *v, const double *const *e, double *kinetic,
+                 double *internal) {
+  int rc;
+  std::vector<blast_cf *> hs(n);
+  std::vector<double *> ap(n), out(n);
+  for (int r = 0; r < n; ++r) {
+    blast_cf_rk2 *s = S[r];
+    hs[r] = s->h; ap[r] = s->AP; out[r] = s->scal_out;
+    cudaStream_t st = s->hv.stream;
+    CUDA_TRY(cudaMemsetAsync(s->scal_out, 0, 2 * sizeof(double), st));
+    launch_mass_zone(s, v[r], nullptr, nullptr);
+    if (s->hv.nn > 0) {
+      if (s->multi) {   // M_V v to the nodes; its dot with v after the shared-node sum
+        if (s->hv.dim == 3) k_gather<3><<<blocks_for(s->hv.nn, NB), NB, 0, st>>>(node_args(s), s->Y, s->AP);
+        else k_gather<2><<<blocks_for(s->hv.nn, NB), NB, 0, st>>>(node_args(s), s->Y, s->AP);
+      } else if (s->hv.dim == 3) {
+        k_gather_dot<3><<<blocks_for(s->hv.nn, NB), NB, 0, st>>>(node_args(s), s->Y, v[r], s->partials, s->ticket, s->scal_out);
+      } else {
+        k_gather_dot<2><<<blocks_for(s->hv.nn, NB), NB, 0, st>>>(node_args(s), s->Y, v[r], s->partials, s->ticket, s->scal_out);
+      }
+    }
+    if (s->ne > 0) k_dot<<<blocks_for(s->ne, NB), NB, 0, st>>>(s->me1, e[r], s->ne, s->partials, s->ticket, s->scal_out + 1);
+  }
+  if (S[0]->multi) {
+    if ((rc = blastcf::group_exchange_sum(hs.data(), n, ap.data()))) return rc;
+    for (int r = 0; r < n; ++r) {
+      blast_cf_rk2 *s = S[r];
+      if (s->hv.nn == 0) continue;
+      if (s->hv.dim == 3) k_wdot<3><<<blocks_for(s->hv.nn, NB), NB, 0, s->hv.stream>>>(s->hv.nn, v[r], s->AP, s->own, s->partials, s->ticket, s->scal_out);
+      else k_wdot<2><<<blocks_for(s->hv.nn, NB), NB, 0, s->hv.stream>>>(s->hv.nn, v[r], s->AP, s->own, s->partials, s->ticket, s->scal_out);
+    }
+    if ((rc = blastcf::group_allreduce(hs.data(), n, out.data(), 2, 0))) return rc;
+  }
+  if ((rc = check("energy"))) return rc;
+  double res[2];
+  CUDA_TRY(cudaMemcpyAsync(res, S[0]->scal_out, sizeof res, cudaMemcpyDeviceToHost, S[0]->hv.stream));
+  for (int r = 0; r < n; ++r) CUDA_TRY(cudaStreamSynchronize(S[r]->hv.stream));
+  *kinetic = 0.5 * res[0];
+  *internal = res[1];
+  return BLAST_CF_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -657,6 +905,7 @@ void blast_cf_rk2_default_opts(blast_cf_rk2_opts *o) {
   o->cg_max_iter = 500;
   o->cg_check_every = 8;
   o->wall_bc = 1;
+  for (int c = 0; c < 3; ++c) o->box_lo[c] = o->box_hi[c] = 0.0;   // not given: derived at create
 }
 
 int blast_cf_rk2_create(blast_cf *h, const blast_cf_mesh *mesh, const double *rho0detJ0,
@@ -670,7 +919,8 @@ int blast_cf_rk2_create(blast_cf *h, const blast_cf_mesh *mesh, const double *rh
   int rc = blastcf::handle_view(h, &s->hv);
   if (rc) return bail(rc);
   const HandleView &hv = s->hv;
-  if (hv.multi_rank) return bail(fail(BLAST_CF_EUNSUPPORTED, "the integrator is single-GPU (nranks == 1) in this version"));
+  s->multi = hv.multi_rank;
+  s->loopback = hv.loopback;
   if (mesh->num_zones != hv.Z || mesh->num_nodes != hv.nn || mesh->dim != hv.dim || mesh->order != hv.k)
     return bail(fail(BLAST_CF_EINVAL, "mesh does not match the handle"));
   if (hv.Z > 0 && !rho0detJ0) return bail(fail(BLAST_CF_EINVAL, "rho0detJ0 is NULL"));
@@ -718,6 +968,13 @@ int blast_cf_rk2_create(blast_cf *h, const blast_cf_mesh *mesh, const double *rh
   CUDA_TRY(cudaMalloc(&s->sc, sizeof(CGScal)));
   CUDA_TRY(cudaMemset(s->sc, 0, sizeof(CGScal)));
   CUDA_TRY(cudaMallocHost(&s->h_sc, sizeof(CGScal)));
+  CUDA_TRY(cudaMalloc(&s->red, (2 * D + 2) * sizeof(double)));
+  if (s->multi) {
+    std::vector<double> own(std::max<int64_t>(nn, 1), 1.0);
+    if ((rc = blastcf::owner_weights(h, own.data()))) return bail(rc);
+    CUDA_TRY(cudaMalloc(&s->own, own.size() * sizeof(double)));
+    CUDA_TRY(cudaMemcpy(s->own, own.data(), own.size() * sizeof(double), cudaMemcpyHostToDevice));
+  }
   CUDA_TRY(cudaMalloc(&s->m1inv, (size_t)t * t * sizeof(double)));
   CUDA_TRY(cudaMalloc(&s->zscale, std::max<int64_t>(Z, 1) * sizeof(double)));
   if (Z > 0) CUDA_TRY(cudaMemcpy(s->R, rho0detJ0, (size_t)Z * hv.nq * sizeof(double), cudaMemcpyHostToDevice));
@@ -801,22 +1058,41 @@ int blast_cf_rk2_create(blast_cf *h, const blast_cf_mesh *mesh, const double *rh
     else k_gather<2><<<blocks_for(nn, NB), NB, 0, st>>>(node_args(s), s->Y, s->invd);
   }
   if ((rc = check("create kernels"))) return bail(rc);
-  std::vector<double> diag(nx, 0.0);
-  if (nn > 0) CUDA_TRY(cudaMemcpyAsync(diag.data(), s->invd, s->nx * sizeof(double), cudaMemcpyDeviceToHost, st));
-  CUDA_TRY(cudaStreamSynchronize(st));
+  // walls (reading R23): the faces of the GLOBAL box.  Given in opts, else the bounding box of x0 (one
+  // rank) or its group min / max (NCCL ranks); a loopback group must pass it (no collective at create).
+  double lo[3], hi[3];
+  const bool given = s->opts.box_hi[0] > s->opts.box_lo[0];
   for (int c = 0; c < D; ++c) {
-    double lo = HUGE_VAL, hi = -HUGE_VAL;
-    for (int64_t i = 0; i < nn; ++i) { lo = std::min(lo, mesh->x0[c * nn + i]); hi = std::max(hi, mesh->x0[c * nn + i]); }
-    const double tol = 1e-12 * (hi - lo);
+    lo[c] = given ? s->opts.box_lo[c] : HUGE_VAL;
+    hi[c] = given ? s->opts.box_hi[c] : -HUGE_VAL;
+    for (int64_t i = 0; i < nn && !given; ++i) { lo[c] = std::min(lo[c], mesh->x0[c * nn + i]); hi[c] = std::max(hi[c], mesh->x0[c * nn + i]); }
+  }
+  if (s->multi && !given && s->opts.wall_bc) {
+    if (s->loopback) return bail(fail(BLAST_CF_EINVAL, "a loopback group needs opts->box_lo/box_hi (the global box)"));
+    double mm[6] = {0, 0, 0, 0, 0, 0};
+    for (int c = 0; c < D; ++c) { mm[c] = -lo[c]; mm[3 + c] = hi[c]; }
+    CUDA_TRY(cudaMemcpy(s->red, mm, 6 * sizeof(double), cudaMemcpyHostToDevice));
+    blast_cf *hh = h;
+    double *rb = s->red;
+    if ((rc = blastcf::group_allreduce(&hh, 1, &rb, 6, 2))) return bail(rc);
+    CUDA_TRY(cudaStreamSynchronize(st));
+    CUDA_TRY(cudaMemcpy(mm, s->red, 6 * sizeof(double), cudaMemcpyDeviceToHost));
+    for (int c = 0; c < D; ++c) { lo[c] = -mm[c]; hi[c] = mm[3 + c]; }
+  }
+  s->fixed.assign(nx, 0);
+  for (int c = 0; c < D; ++c) {
+    const double tol = 1e-12 * (hi[c] - lo[c]);
     for (int64_t i = 0; i < nn; ++i) {
       const double xv = mesh->x0[c * nn + i];
-      const bool fixed = s->opts.wall_bc && (fabs(xv - lo) <= tol || fabs(xv - hi) <= tol);
-      double &d = diag[c * nn + i];
-      if (!(d > 0.0) && !fixed) return bail(fail(BLAST_CF_EINVAL, "non-positive mass diagonal at node %lld", (long long)i));
-      d = fixed ? 0.0 : 1.0 / d;
+      s->fixed[c * nn + i] = s->opts.wall_bc && (fabs(xv - lo[c]) <= tol || fabs(xv - hi[c]) <= tol);
     }
   }
-  if (nn > 0) CUDA_TRY(cudaMemcpy(s->invd, diag.data(), s->nx * sizeof(double), cudaMemcpyHostToDevice));
+  // the Jacobi diagonal: shared-node sum first (a partition's zones give only part of a shared node's
+  // diagonal), then inverted with the wall mask; a loopback group does that in blast_cf_rk2_setup_loopback
+  if (!s->loopback) {
+    blast_cf_rk2 *one = s;
+    if ((rc = finish_setup(&one, 1))) return bail(rc);
+  }
   *out = s;
   return BLAST_CF_OK;
 }
@@ -824,34 +1100,54 @@ int blast_cf_rk2_create(blast_cf *h, const blast_cf_mesh *mesh, const double *rh
 int blast_cf_rk2_rates(blast_cf_rk2 *s, const double *x, const double *v, const double *e, const double *vbar,
                        double *out_dvdt, double *out_dedt, double *out_dt, int32_t *cg_iters) {
   if (!s || !out_dvdt || !out_dedt) return fail(BLAST_CF_EINVAL, "NULL argument");
-  int rc = blastcf::eval_with_S(s->h, x, v, e, s->R, s->F1, s->FTv, s->dtd, s->Sq);
-  if (rc) return rc;
-  int it = 0;
-  if ((rc = cg_solve(s, s->F1, -1.0, out_dvdt, &it))) return rc;
-  if (cg_iters) *cg_iters = it;
-  launch_energy_rhs(s, vbar ? vbar : v, out_dedt);
-  if ((rc = check("energy rhs"))) return rc;
-  if (out_dt) CUDA_TRY(cudaMemcpyAsync(out_dt, s->dtd, sizeof(double), cudaMemcpyDeviceToHost, s->hv.stream));
-  CUDA_TRY(cudaStreamSynchronize(s->hv.stream));
-  return BLAST_CF_OK;
+  if (s->loopback) return fail(BLAST_CF_EINVAL, "loopback group: use blast_cf_rk2_rates_loopback");
+  return rates_group(&s, 1, &x, &v, &e, &vbar, &out_dvdt, &out_dedt, out_dt, cg_iters);
+}
+
+int blast_cf_rk2_rates_loopback(blast_cf_rk2 *const *S, int n, const double *const *x, const double *const *v,
+                                const double *const *e, const double *const *vbar, double *const *out_dvdt,
+                                double *const *out_dedt, double *out_dt, int32_t *cg_iters) {
+  if (!S || n < 1 || !x || !v || !e || !out_dvdt || !out_dedt) return fail(BLAST_CF_EINVAL, "NULL argument");
+  for (int r = 0; r < n; ++r)
+    if (!S[r] || !S[r]->loopback || S[r]->hv.rank != r || S[r]->hv.nranks != n || !S[r]->ready)
+      return fail(BLAST_CF_EINVAL, "integrator %d is not rank %d of a set-up %d-rank loopback group", r, r, n);
+  return rates_group(S, n, x, v, e, vbar, out_dvdt, out_dedt, out_dt, cg_iters);
+}
+
+int blast_cf_rk2_setup_loopback(blast_cf_rk2 *const *S, int n) {
+  if (!S || n < 1) return fail(BLAST_CF_EINVAL, "NULL argument");
+  for (int r = 0; r < n; ++r)
+    if (!S[r] || !S[r]->loopback || S[r]->hv.rank != r || S[r]->hv.nranks != n)
+      return fail(BLAST_CF_EINVAL, "integrator %d is not rank %d of a %d-rank loopback group", r, r, n);
+  return finish_setup(S, n);
+}
+
+int blast_cf_rk2_energy_loopback(blast_cf_rk2 *const *S, int n, const double *const *v, const double *const *e,
+                                 double *kinetic, double *internal) {
+  if (!S || n < 1 || !v || !e || !kinetic || !internal) return fail(BLAST_CF_EINVAL, "NULL argument");
+  for (int r = 0; r < n; ++r)
+    if (!S[r] || !S[r]->loopback || S[r]->hv.rank != r || S[r]->hv.nranks != n)
+      return fail(BLAST_CF_EINVAL, "integrator %d is not rank %d of a %d-rank loopback group", r, r, n);
+  return energy_group(S, n, v, e, kinetic, internal);
 }
 
 int blast_cf_rk2_step(blast_cf_rk2 *s, double *x, double *v, double *e, double dt, double *dt_est,
                       int32_t *cg_iters) {
   if (!s || ((!x || !v) && s->nx > 0) || (!e && s->ne > 0)) return fail(BLAST_CF_EINVAL, "NULL argument");
+  if (s->loopback) return fail(BLAST_CF_EINVAL, "loopback group: step the ranks with blast_cf_rk2_rates_loopback");
   const double h = 0.5 * dt;
   int rc, it0 = 0, it1 = 0;
   cudaStream_t st = s->hv.stream;
   // stage 1 at S0
   if ((rc = blastcf::eval_with_S(s->h, x, v, e, s->R, s->F1, s->FTv, s->dtd, s->Sq))) return rc;
-  if ((rc = cg_solve(s, s->F1, -1.0, s->DV, &it0))) return rc;
+  if ((rc = cg_group(&s, 1, &s->F1, -1.0, &s->DV, &it0))) return rc;
   axpy(s, s->Vb, v, h, s->DV, s->nx);                    // Vb = v0 + dt/2 dv0
   launch_energy_rhs(s, s->Vb, s->DE);                    // de0 = M_E^{-1} F(S0)^T Vb
   axpy(s, s->xh, x, h, s->Vb, s->nx);                    // x_half
   axpy(s, s->eh, e, h, s->DE, s->ne);                    // e_half
   // stage 2 at S_half = (x_half, Vb, e_half)
   if ((rc = blastcf::eval_with_S(s->h, s->xh, s->Vb, s->eh, s->R, s->F1, s->FTv, s->dtd + 1, s->Sq))) return rc;
-  if ((rc = cg_solve(s, s->F1, -1.0, s->DV, &it1))) return rc;
+  if ((rc = cg_group(&s, 1, &s->F1, -1.0, &s->DV, &it1))) return rc;
   axpy(s, s->Vb, v, h, s->DV, s->nx);                    // Vb = v0 + dt/2 dv1
   launch_energy_rhs(s, s->Vb, s->DE);                    // de1
   axpy(s, x, x, dt, s->Vb, s->nx);
@@ -918,24 +1214,8 @@ int blast_cf_rk2_mass_apply(blast_cf_rk2 *s, const double *u, double *out) {
 
 int blast_cf_rk2_energy(blast_cf_rk2 *s, const double *v, const double *e, double *kinetic, double *internal) {
   if (!s || !kinetic || !internal) return fail(BLAST_CF_EINVAL, "NULL argument");
-  cudaStream_t st = s->hv.stream;
-  CUDA_TRY(cudaMemsetAsync(s->scal_out, 0, 2 * sizeof(double), st));
-  launch_mass_zone(s, v, nullptr, nullptr);
-  if (s->hv.nn > 0) {
-    if (s->hv.dim == 3)
-      k_gather_dot<3><<<blocks_for(s->hv.nn, NB), NB, 0, st>>>(node_args(s), s->Y, v, s->partials, s->ticket, s->scal_out);
-    else
-      k_gather_dot<2><<<blocks_for(s->hv.nn, NB), NB, 0, st>>>(node_args(s), s->Y, v, s->partials, s->ticket, s->scal_out);
-  }
-  if (s->ne > 0) k_dot<<<blocks_for(s->ne, NB), NB, 0, st>>>(s->me1, e, s->ne, s->partials, s->ticket, s->scal_out + 1);
-  int rc = check("energy");
-  if (rc) return rc;
-  double r[2];
-  CUDA_TRY(cudaMemcpyAsync(r, s->scal_out, sizeof r, cudaMemcpyDeviceToHost, st));
-  CUDA_TRY(cudaStreamSynchronize(st));
-  *kinetic = 0.5 * r[0];
-  *internal = r[1];
-  return BLAST_CF_OK;
+  if (s->loopback) return fail(BLAST_CF_EINVAL, "loopback group: use blast_cf_rk2_energy_loopback");
+  return energy_group(&s, 1, &v, &e, kinetic, internal);
 }
 
 int blast_cf_rk2_destroy(blast_cf_rk2 *s) {

@@ -174,7 +174,8 @@ def test_quiescent_box_gpu(orc):
     assert float(v.abs().max()) < 1e-13 and float((e - 2.0).abs().max()) < 1e-13
 
 
-def test_multi_rank_handle_rejected(orc):
+def test_loopback_integrator_needs_global_box(orc):
+    """A loopback rank cannot find the global walls by itself (no collective at create): EINVAL."""
     torch = _torch()
     import paper_conf_ipps_dongdkrtd14_b200 as cf
     import oracle

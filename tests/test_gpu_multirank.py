@@ -46,3 +46,50 @@ def test_loopback_exchange(orc, name, N, k, P):
     for p, (f1, _, _) in zip(parts, outs):
         glob[:, p.nodes] = f1.cpu().numpy()
     assert np.abs(glob - r.F1).max() <= 1e-12 * np.abs(r.F1).max()
+
+
+@pytest.mark.parametrize("name,N,k,P", [("C3", (4, 4, 4), None, 2), ("C3", (4, 4, 4), None, 8),
+                                        ("C2", (8, 6), 3, 4), ("C5", (4, 2, 2), 2, 8)])
+def test_loopback_integrator(name, N, k, P):
+    """Multi-GPU CG for M_V on one GPU: every rank of a loopback group runs the group
+    CG (shared-node sum of A p each iteration, owner-weighted dot products summed over the ranks) inside
+    blast_cf_rk2_rates_loopback; dv/dt, de/dt, dt and the energies must match the single-domain
+    integrator, and every sharer of a node must hold the same bits."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import ctypes
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    m, s = synth.config(name, "S1", N=N, k=k)
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    h1 = cf.from_synth(m)
+    r1 = cf.RK2(h1, s.rho0detJ0, cg_rel_tol=1e-15)
+    x, v, e = t(s.x), t(s.v), t(s.e)
+    dv1, de1, dt1, it1 = (a.cpu().numpy() if hasattr(a, "cpu") else a for a in r1.rates(x, v, e))
+    ke1, ie1 = r1.energy(v, e)
+    par = cf.default_params()
+    par.h0 = h1.info["h0"]
+    parts = synth.partition(m, P)
+    box = dict(box_lo=(ctypes.c_double * 3)(*([0.0] * 3)),
+               box_hi=(ctypes.c_double * 3)(*(list(m.L) + [0.0] * (3 - m.dim))))
+    hs = [cf.from_synth(m, params=par, part=p, nccl_uid=None) for p in parts]
+    ls = [p.local_state(s) for p in parts]
+    rk = [cf.RK2(h, l.rho0detJ0, cg_rel_tol=1e-15, **box) for h, l in zip(hs, ls)]
+    cf.rk2_setup_loopback(rk)
+    xs, vs, es = [t(l.x) for l in ls], [t(l.v) for l in ls], [t(l.e) for l in ls]
+    dvs, des, dt, it = cf.rk2_rates_loopback(rk, xs, vs, es)
+    ke, ie = cf.rk2_energy_loopback(rk, vs, es)
+    assert dt == dt1
+    assert abs(it - it1) <= 3, (it, it1)
+    sdv, sde = np.abs(dv1).max(), np.abs(de1).max()
+    shared = {}
+    for p, dv, de in zip(parts, dvs, des):
+        dv, de = dv.cpu().numpy(), de.cpu().numpy()
+        assert np.abs(dv - dv1[:, p.nodes]).max() <= 1e-11 * sdv
+        assert np.abs(de - de1[p.zones]).max() <= 1e-12 * sde
+        for g, val in zip(p.nodes, dv.T):
+            if g in shared:
+                assert np.array_equal(shared[g], val)   # every sharer holds the same iterate bits
+            else:
+                shared[g] = val
+    assert abs(ke - ke1) <= 1e-13 * max(abs(ke1), 1e-300) and abs(ie - ie1) <= 1e-13 * abs(ie1)
