@@ -287,8 +287,8 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
 #pragma unroll
               for (int c5 = 0; c5 < 5; ++c5) {
                 const int cd = h * 5 + c5;
-                if (cd < 9 && lr < P) Wr[Dm::O_Y + (cd * P + lr) * N2 + col] = d[c5][i];
-                if (cd == 9 && lr < T) Wr[Dm::O_YE + lr * N2 + col] = d[c5][i];
+                if (cd < 9 && lr < P) Wr[Dm::O_Y + (cd * P + lr) * Dm::YS + col] = d[c5][i];
+                if (cd == 9 && lr < T) Wr[Dm::O_YE + lr * Dm::YS + col] = d[c5][i];
               }
             }
           }
@@ -308,13 +308,13 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
           const int c = j / NTL, tl = j - c * NTL;
           const int nb = min(tl * 8 + lr, NC - 1);
           const int q2b = nb / P, a0b = nb - q2b * P;
-          const double *Yb = Wr + Dm::O_Y + (c * 3 * P + a0b) * N2 + q2b * N;
+          const double *Yb = Wr + Dm::O_Y + (c * 3 * P + a0b) * Dm::YS + q2b * N;
 #pragma unroll
           for (int s = 0; s < KS_N; ++s) {
             const int q1 = min(4 * s + lc, N - 1);
             y[t][0][s] = Yb[q1];
-            y[t][1][s] = Yb[P * N2 + q1];
-            y[t][2][s] = Yb[2 * P * N2 + q1];
+            y[t][1][s] = Yb[P * Dm::YS + q1];
+            y[t][2][s] = Yb[2 * P * Dm::YS + q1];
           }
         }
         double zb[JPW][2], zg[JPW][2];
@@ -349,7 +349,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
         const int q2b = nb / T, j0b = nb - q2b * T;
         double d0 = 0.0, d1 = 0.0;
 #pragma unroll
-        for (int s = 0; s < KS_N; ++s) dmma(d0, d1, fPt[s], Wr[Dm::O_YE + j0b * N2 + q2b * N + min(4 * s + lc, N - 1)]);
+        for (int s = 0; s < KS_N; ++s) dmma(d0, d1, fPt[s], Wr[Dm::O_YE + j0b * Dm::YS + q2b * N + min(4 * s + lc, N - 1)]);
 #pragma unroll
         for (int i = 0; i < 2; ++i) {
           const int n = te * 8 + 2 * lc + i;

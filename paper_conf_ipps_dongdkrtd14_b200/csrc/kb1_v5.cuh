@@ -30,7 +30,10 @@ struct V5Dims {
   // KW scratch: XE (X[6][P^3] E[T^3] J0[9] gamma, cp.async) | forward T/TE + UX | back Y/YE + Z/ZE
   static constexpr int XE_X = 0, XE_E = 6 * P3, XE_J = XE_E + T3, XE = (XE_J + 10 + 1) / 2 * 2;
   static constexpr int O_T = 0, O_TE = 12 * N * P2, O_UX = (O_TE + N * T2 + 1) / 2 * 2, FWREG = O_UX + 9 * N2 * P;
-  static constexpr int O_Y = 0, O_YE = 9 * P * N2, O_Z = O_YE + T * N2, O_ZE = O_Z + 6 * N * P2;
+  // Y / YE rows (one per (component, a0) / j0) are YS = N^2 + 4 apart: kb1_v10's DMMA C^T stores and B^T
+  // loads put 5 rows in one warp access, which a stride of N^2 = 64 maps onto the same banks (5-way)
+  static constexpr int YS = N2 + 4;
+  static constexpr int O_Y = 0, O_YE = 9 * P * YS, O_Z = O_YE + T * YS, O_ZE = O_Z + 6 * N * P2;
   static constexpr int YZREG = O_ZE + N * T2;
   static constexpr int WREG = ((FWREG > YZREG ? FWREG : YZREG) + 1) / 2 * 2;
   // totals (every region starts on a 16-byte boundary)
