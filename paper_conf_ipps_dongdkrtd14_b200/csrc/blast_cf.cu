@@ -134,16 +134,16 @@ KB1Variant variant3v6() {
   using C = KB1V5Cfg<K>;
   return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v6<K, DIAG>, (const void *)&kb1_v6_3d<K, DIAG>, true, nullptr};
 }
-template <int K, int DIAG, int MODE, int OPT>
+template <int K, int DIAG, int MODE, int OPT, int VMODE>
 void launch3v10(const KB1Args &a, int grid, cudaStream_t s) {
   using C = KB1V5Cfg<K, MODE>;
-  kb1_v10_3d<K, DIAG, MODE, OPT><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+  kb1_v10_3d<K, DIAG, MODE, OPT, VMODE><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
 }
-template <int K, int DIAG = 0, int MODE = 0, int OPT = 0>
+template <int K, int DIAG = 0, int MODE = 0, int OPT = 0, int VMODE = 0>
 KB1Variant variant3v10() {
   using C = KB1V5Cfg<K, MODE>;
-  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v10<K, DIAG, MODE, OPT>,
-                    (const void *)&kb1_v10_3d<K, DIAG, MODE, OPT>, true, nullptr};
+  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v10<K, DIAG, MODE, OPT, VMODE>,
+                    (const void *)&kb1_v10_3d<K, DIAG, MODE, OPT, VMODE>, true, nullptr};
 }
 template <int K, int MINB>
 void launch3v8(const KB1Args &a, int grid, cudaStream_t s) {
@@ -179,7 +179,7 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
       case 2: add(variant3v2<2, 4, 3>(), "v2.z4"); add(variant3v2<2, 4, 2, 1>(), "v2.p1.z4"); add(variant3v2<2, 2, 4, 1>(), "v2.p1.z2"); add(variant3v3<2, 4, 2>(), "v3.z4"); add(variant3<2, 16, 2>(), "v1.z16"); break;
       case 3: add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3v2<3, 1, 2, 1>(), "v2.p1.z1"); add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
       case 4:
-        add(variant3v10<4>(), "v10"); add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
+        add(variant3v10<4, 0, 0, 0, 3>(), "v10.w"); add(variant3v10<4, 0, 0, 0, 2>(), "v10.v"); add(variant3v10<4>(), "v10"); add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
@@ -192,7 +192,7 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
       case 1: add(variant2<1, 64, 2>(), "v1-2d.z64"); break;
       case 2: add(variant2<2, 16, 2>(), "v1-2d.z16"); break;
       case 3: add(variant2<3, 8, 2>(), "v1-2d.z8"); break;
-      case 4: add(variant2<4, 4, 2>(), "v1-2d.z4"); break;
+      case 4: add(variant2<4, 4, 3>(), "v1-2d.z4m3"); add(variant2<4, 4, 2>(), "v1-2d.z4"); add(variant2<4, 2, 4>(), "v1-2d.z2m4"); break;
       case 5: add(variant2<5, 2, 2>(), "v1-2d.z2"); break;
       case 6: add(variant2<6, 2, 2>(), "v1-2d.z2"); break;
       case 7: add(variant2<7, 1, 2>(), "v1-2d.z1"); break;
@@ -219,6 +219,9 @@ KB1Variant select_variant(int dim, int k) {
       if (strcmp(force, "v10.q") == 0) { d = variant3v10<4, 0, 0, 4>(); d.name = "v10.q"; return d; }
       if (strcmp(force, "v10.b") == 0) { d = variant3v10<4, 0, 0, 1>(); d.name = "v10.b"; return d; }
       if (strcmp(force, "v10.l") == 0) { d = variant3v10<4, 0, 0, 2>(); d.name = "v10.l"; return d; }
+      if (strcmp(force, "v10.wr3") == 0) { d = variant3v10<4, 0, 3, 0, 3>(); d.name = "v10.wr3"; return d; }
+      if (strcmp(force, "v10.wd1") == 0) { d = variant3v10<4, 1, 0, 0, 3>(); d.name = "v10.wd1"; return d; }
+      if (strcmp(force, "v10.vd1") == 0) { d = variant3v10<4, 1, 0, 0, 2>(); d.name = "v10.vd1"; return d; }
       if (strcmp(force, "v10.d1") == 0) { d = variant3v10<4, 1>(); d.name = "v10.d1"; return d; }
       if (strcmp(force, "v10.d2") == 0) { d = variant3v10<4, 2>(); d.name = "v10.d2"; return d; }
       if (strcmp(force, "v5.r2") == 0) { d = variant3v5<4, 0, 2>(); d.name = "v5.r2"; return d; }

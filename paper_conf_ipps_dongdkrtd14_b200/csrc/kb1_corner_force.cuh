@@ -371,6 +371,14 @@ __global__ void __launch_bounds__(KB1Cfg2<K, ZPC>::NTH, MINB) kb1_corner_force_2
   const int64_t Z = a.num_zones, nn = a.num_nodes;
 
   for (int i = tid; i < Dm::TAB; i += NTH) smem[i] = a.tab[i];
+  // the point stage's global operands (rho0|J0| of this thread's point, gamma of its zone) are loaded
+  // here, so their DRAM latency overlaps the gather instead of stalling the point stage
+  const int my_zl = tid / NQ, my_q = tid - my_zl * NQ;
+  const bool has_point = my_zl < ZPC;
+  const int64_t my_z = zone0 + my_zl;
+  const bool active = has_point && my_z < Z;
+  const double Rq = active ? __ldg(a.rho0detJ0 + my_z * NQ + my_q) : 1.0;
+  const double gamma_z = active ? __ldg(a.zone_gamma + my_z) : 1.4;
   for (int i = tid; i < ZPC * NK; i += NTH) {
     const int zl = i / NK, r = i - zl * NK;
     const int64_t z = zone0 + zl;
@@ -422,11 +430,7 @@ __global__ void __launch_bounds__(KB1Cfg2<K, ZPC>::NTH, MINB) kb1_corner_force_2
     sT[zl * Dm::SZ_T + 2 * NF * N * P + r] = te;
   }
   __syncthreads();
-  const int my_zl = tid / NQ, my_q = tid - my_zl * NQ;
   const int q0 = my_q % N, q1 = my_q / N;
-  const bool has_point = my_zl < ZPC;
-  const int64_t my_z = zone0 + my_zl;
-  const bool active = has_point && my_z < Z;
   double dtmin = __longlong_as_double(0x7ff0000000000000LL);
   bool bad = false;
   if (has_point) {
@@ -447,11 +451,9 @@ __global__ void __launch_bounds__(KB1Cfg2<K, ZPC>::NTH, MINB) kb1_corner_force_2
     double eq = 0.0;
 #pragma unroll
     for (int j0 = 0; j0 < T; ++j0) eq = fma(sPhi[q0 * T + j0], Tz[2 * NF * N * P + q1 * T + j0], eq);
-    const double R = active ? __ldg(a.rho0detJ0 + my_z * NQ + my_q) : 1.0;
-    const double gamma = active ? __ldg(a.zone_gamma + my_z) : 1.4;
     const double alpha = sW[q0] * sW[q1];
     PointOut<2> o;
-    point_eval2(Jm, Gv, eq, R, alpha, gamma, sJ0 + my_zl * 4, a.ph, o);
+    point_eval2(Jm, Gv, eq, Rq, alpha, gamma_z, sJ0 + my_zl * 4, a.ph, o);
     double *S = sS + my_zl * Dm::SZ_S;
 #pragma unroll
     for (int c = 0; c < 2; ++c)

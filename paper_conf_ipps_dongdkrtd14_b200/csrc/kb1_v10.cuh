@@ -37,7 +37,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned parity) {
       : "memory");
 }
 
-template <int K, int DIAG = 0, int MODE = 0, int OPT = 0>
+template <int K, int DIAG = 0, int MODE = 0, int OPT = 0, int VMODE = 0>
 __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB1Args a) {
   using Dm = V5Dims<K>;
   using Cfg = KB1V5Cfg<K, MODE>;
@@ -465,8 +465,25 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     const double w12 = sW[q1] * sW[q2];
     PointOut<3> oa, ob;
     const double best = sRed[8];   // largest exact inverse dt found so far by this CTA (dt filter)
-    point_eval3<true>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best);
-    point_eval3<true>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best);
+    if (VMODE == 3 && a.ph.use_visc && a.ph.use_vort) {   // both points one straight-line block, one vote
+      point_eval3<2, 1>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best);
+      point_eval3<2, 1>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best);
+      if (__any_sync(0xffffffffu, oa.cand || ob.cand)) {   // J is still in the JS buffer (S is written below)
+        double Jr[3][3];
+#pragma unroll
+        for (int cd = 0; cd < 9; ++cd) Jr[cd / 3][cd % 3] = jb[cd * N3 + sa];
+        point_dt_exact(Jr, a.ph, oa);
+#pragma unroll
+        for (int cd = 0; cd < 9; ++cd) Jr[cd / 3][cd % 3] = jb[cd * N3 + sbi];
+        point_dt_exact(Jr, a.ph, ob);
+      }
+    } else if (VMODE == 1 || (VMODE >= 2 && a.ph.use_visc && a.ph.use_vort)) {   // production switches
+      point_eval3<true, 1>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best);
+      point_eval3<true, 1>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best);
+    } else {
+      point_eval3<true>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best);
+      point_eval3<true>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best);
+    }
     {
       double mi = fmax(oa.inv, ob.inv);
 #pragma unroll

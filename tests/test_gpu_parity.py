@@ -212,7 +212,7 @@ def test_full_size_sampled(orc, name, which):
     sampled_parity(orc, name, which, n_nodes=24 if name == "C5" else 48, n_zones=8 if name == "C5" else 48)
 
 
-@pytest.mark.parametrize("name", ["v5.r1", "v6", "v4.m0"])
+@pytest.mark.parametrize("name", ["v10.v", "v10", "v5.r1", "v6", "v4.m0"])
 def test_full_size_sampled_c4_variants(orc, name, monkeypatch):
     """The persistent warp-specialized C4 candidates at the bench's size (221 zones per CTA: every stage of
     the zone pipeline, both buffers and the dt filter across zones are exercised)."""
@@ -244,7 +244,7 @@ def test_multi_material_gamma(orc):
 
 CANDIDATES = {1: ["v2.p1.z32", "v2.z64", "v1.z32"], 2: ["v2.z4", "v2.p1.z4", "v2.p1.z2", "v3.z4", "v1.z16"],
               3: ["v2.z2", "v2.p1.z1", "v3.z2", "v1.z8"],
-              4: ["v10", "v5.r1", "v4.m0", "v5", "v6", "v4.m1", "v3.z1", "v2.z1", "v1.z4"],
+              4: ["v10.w", "v10.v", "v10", "v5.r1", "v4.m0", "v5", "v6", "v4.m1", "v3.z1", "v2.z1", "v1.z4"],
               7: ["v8", "v1.z1"], 8: ["v8", "v8.m1", "v1.z1m2", "v1.z1"]}
 
 
@@ -253,6 +253,15 @@ def test_every_kernel_variant(orc, k, name, monkeypatch):
     """Every candidate corner-force kernel (BLAST_CF_KB1 picks it at create) meets the parity bar."""
     monkeypatch.setenv("BLAST_CF_KB1", name)
     m, s = synth.config("C4", "S1", N=(5, 3, 2), k=k)
+    h, _, _ = check(m, s, orc)
+    assert h.variant == name
+
+
+@pytest.mark.parametrize("name", ["v1-2d.z4m3", "v1-2d.z4", "v1-2d.z2m4"])
+def test_every_2d_kernel_variant(orc, name, monkeypatch):
+    """The 2D Q4 candidates (C2's order) meet the parity bar, on a mesh with a partial last zone batch."""
+    monkeypatch.setenv("BLAST_CF_KB1", name)
+    m, s = synth.config("C2", "S1", N=(7, 5), k=4)
     h, _, _ = check(m, s, orc)
     assert h.variant == name
 
