@@ -15,6 +15,10 @@
 // OPT bit 1 (LATE): the gather of zone i+1 is issued after the C^T stage of zone i-1 instead of before it,
 // away from the point warps' stage-C shared-memory burst at the start of every zone.
 // OPT bit 2 (BAL): forward stage B's 32 e items go two each to the 16 threads without a field item.
+// OPT bit 3 (PWG): the POINT warps issue the gather of zone i+2 at the end of their zone i (they finish
+// before the contraction warps, which are the bound), into a second XE buffer; completion reaches the
+// contraction warps through cp.async.mbarrier.arrive on a per-buffer mbarrier, so the contraction warps
+// issue nothing (their issue phase was 2.2 K of 11.7 K cycles per zone next to the point warps).
 #pragma once
 #include "kb1_v6.cuh"
 
@@ -30,6 +34,9 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned by
                    smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
                : "memory");
 }
+__device__ __forceinline__ void cp_async_mbar_arrive(uint64_t *bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(bar)) : "memory");
+}
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned parity) {
   asm volatile(
       "{\n.reg .pred p;\nWAIT_%=:\nmbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n@!p bra WAIT_%=;\n}\n" ::"r"(
@@ -41,7 +48,8 @@ template <int K, int DIAG = 0, int MODE = 0, int OPT = 0, int VMODE = 0>
 __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB1Args a) {
   using Dm = V5Dims<K>;
   using Cfg = KB1V5Cfg<K, MODE>;
-  constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4;
+  constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4, PWG = OPT & 8;
+  static_assert(!(PWG && (BULK || LATE)), "PWG replaces the contraction warps' gather");
   static_assert(!BULK || ((Dm::OFF_XE + Dm::XE_E) % 2 == 0 && (Dm::OFF_UV + Dm::O_R) % 2 == 0 && Dm::UVBUF % 2 == 0 &&
                           (Dm::T3 * 8) % 16 == 0 && (Dm::N3 * 8) % 16 == 0),
                 "bulk copies need 16-byte aligned, 16-byte multiple destinations");
@@ -78,6 +86,15 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   for (int i = tid; i < 2 * N * P + N * T + N; i += Cfg::NTH) sTab[i] = __ldg(a.tab + i);
   if (tid == 0) sRed[8] = 0.0;   // dt filter: best exact inverse dt of this CTA (point_eval3<true>)
 
+  double *const sXEb[2] = {sXE, smem + Dm::OFF_XEB};   // PWG: XE of zone i is sXEb[i & 1]
+  if (PWG) {
+    if (tid == 0) {
+      mbar_init(reinterpret_cast<uint64_t *>(smem + Dm::OFF_MB), NPW);
+      mbar_init(reinterpret_cast<uint64_t *>(smem + Dm::OFF_MB) + 1, NPW);
+      asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    }
+    __syncthreads();
+  }
   // ---------------- KW ----------------
   // node ids travel by cp.async into shared memory one zone ahead (a register copy of an __ldg result
   // would be spilled by the 88-register warps and the spill store would wait for the load)
@@ -119,9 +136,9 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   auto kw_wait_bulk = [&](int64_t i) {
     if (BULK && i < nz) mbar_wait(sMB + (i & 1), (unsigned)((i >> 1) & 1));
   };
-  auto kw_forward = [&](double *ub, double *jb, double *js, int zc) {
+  auto kw_forward = [&](double *ub, double *jb, double *js, int zc, const double *xe) {
     const int kt = opaque_tid() - NPW;
-    if (kt < 10) js[kt] = sXE[Dm::XE_J + kt];
+    if (kt < 10) js[kt] = xe[Dm::XE_J + kt];
     double *Tr = sWk, *UX = sWk + Dm::O_UX;
     // stage A: a2 -> q2 (T_B, T_G of the 6 fields; TE of e)
     {
@@ -135,7 +152,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
         const int f = r / P2, aa = r - f * P2;
         double xv[P];
 #pragma unroll
-        for (int a2 = 0; a2 < P; ++a2) xv[a2] = sXE[Dm::XE_X + f * P3 + a2 * P2 + aa];
+        for (int a2 = 0; a2 < P; ++a2) xv[a2] = xe[Dm::XE_X + f * P3 + a2 * P2 + aa];
         double *TB = Tr + Dm::O_T + (f * 2 + 0) * N * P2 + aa, *TG = TB + N * P2;
 #pragma unroll
         for (int q2 = 0; q2 < N; ++q2) {
@@ -152,7 +169,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
         const int jj = r - 6 * P2;
         double ev[T];
 #pragma unroll
-        for (int j2 = 0; j2 < T; ++j2) ev[j2] = sXE[Dm::XE_E + j2 * T2 + jj];
+        for (int j2 = 0; j2 < T; ++j2) ev[j2] = xe[Dm::XE_E + j2 * T2 + jj];
 #pragma unroll
         for (int q2 = 0; q2 < N; ++q2) {
           double te = 0.0;
@@ -520,17 +537,21 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       mbar_init(sMB + 1, 1);
       asm volatile("fence.mbarrier_init.release.cluster;\nfence.proxy.async.shared::cta;\n" ::: "memory");
     }
-    kw_load_id(0);
-    cp_async_commit();
-    cp_async_wait<0>();
-    kw_bar<NKW>();                   // ids of zone 0 (and the mbarrier init)
-    kw_issue(0);
-    kw_load_id(1);
-    cp_async_commit();
-    cp_async_wait<0>();
-    kw_wait_bulk(0);
+    if (PWG) {   // the point warps issue the gathers
+      if (nz > 0) mbar_wait(sMB, 0u);
+    } else {
+      kw_load_id(0);
+      cp_async_commit();
+      cp_async_wait<0>();
+      kw_bar<NKW>();                 // ids of zone 0 (and the mbarrier init)
+      kw_issue(0);
+      kw_load_id(1);
+      cp_async_commit();
+      cp_async_wait<0>();
+      kw_wait_bulk(0);
+    }
     kw_bar<NKW>();
-    if (nz > 0 && DIAG != 1) kw_forward(sUV, sJS, sJ, a.zero);
+    if (nz > 0 && DIAG != 1) kw_forward(sUV, sJS, sJ, a.zero, sXEb[0]);
     __syncthreads();
     long long t_work = 0;
     int itc = 2;
@@ -542,16 +563,21 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
         cp_async_commit();
       };
       const bool back = i >= 1 && DIAG != 1;
-      if (!(LATE && back)) issue();
+      if (!PWG && !(LATE && back)) issue();
       kstamp(3);
       const int zc = a.zero * itc;   // 0, but loop-variant and uniform
       if (back) kw_back(sJS + ((i - 1) & 1) * Dm::JSBUF, zone_of(i - 1), zc, [&] { if (LATE) issue(); });
-      cp_async_wait<0>();
-      kw_wait_bulk(i + 1);
+      if (PWG) {
+        if (i + 1 < nz) mbar_wait(sMB + ((i + 1) & 1), (unsigned)(((i + 1) >> 1) & 1));
+      } else {
+        cp_async_wait<0>();
+        kw_wait_bulk(i + 1);
+      }
       kw_bar<NKW>();
       kstamp(7);
       if (i + 1 < nz && DIAG != 1)
-        kw_forward(sUV + ((i + 1) & 1) * Dm::UVBUF, sJS + ((i + 1) & 1) * Dm::JSBUF, sJ + ((i + 1) & 1) * 10, zc + a.zero);
+        kw_forward(sUV + ((i + 1) & 1) * Dm::UVBUF, sJS + ((i + 1) & 1) * Dm::JSBUF, sJ + ((i + 1) & 1) * 10, zc + a.zero,
+                   PWG ? sXEb[(i + 1) & 1] : sXE);
       t_work += clock64() - t0;
       __syncthreads();
       kstamp(11);
@@ -563,15 +589,62 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     return;
   }
   asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;\n" ::"n"(Cfg::REG_PW));
+  // PWG: the gather of zone zi (node ids one zone earlier), issued by the point warps; every point thread
+  // arrives once per zone on mbarrier zi & 1 when its copies have landed.  A thread copies rho0|J0| of
+  // exactly its own two points, so it never overwrites an entry another thread has still to read.
+  auto pw_load_id = [&](int64_t zi) {
+    if (zi < nz && tid < P3) cp_async4(sID + (zi & 1) * P3 + tid, a.zone_nodes + zone_of(zi) * P3 + tid);
+  };
+  auto pw_issue = [&](int64_t zi) {
+    if (zi >= nz) return;
+    const int64_t z = zone_of(zi);
+    double *xe = sXEb[zi & 1];
+    if (tid < P3) {
+      const int64_t node = sID[(zi & 1) * P3 + tid];
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        cp_async8(xe + Dm::XE_X + c * P3 + tid, a.x + c * nn + node, true);
+        cp_async8(xe + Dm::XE_X + (3 + c) * P3 + tid, a.v + c * nn + node, true);
+      }
+    } else if (tid < P3 + T3 + 10) {
+      const int r = tid - P3;
+      const double *src = r < T3 ? a.e + z * T3 + r : r < T3 + 9 ? a.J0inv + z * 9 + (r - T3) : a.zone_gamma + z;
+      cp_async8(xe + Dm::XE_E + r, src, true);
+    }
+    if (tid < TPZ) {
+      const int qa = (q2 * N + q1) * N + q0a;
+      double *R = sUV + (zi & 1) * Dm::UVBUF + Dm::O_R;
+      cp_async8(R + qa, a.rho0detJ0 + z * N3 + qa, true);
+      cp_async8(R + qa + NH, a.rho0detJ0 + z * N3 + qa + NH, true);
+    }
+    cp_async_mbar_arrive(sMB + (zi & 1));
+  };
+  if (PWG) {
+    pw_load_id(0);
+    pw_load_id(1);
+    cp_async_commit();
+    cp_async_wait<0>();   // each thread reads back only the ids it loaded
+    pw_issue(0);
+    pw_issue(1);
+    pw_load_id(2);
+    cp_async_commit();
+  }
   __syncthreads();
   long long t_work = 0, t_all = clock64();
   for (int64_t i = 0; i <= nz; ++i) {
     const long long t0 = clock64();
     if (i < nz && tid < TPZ && DIAG != 2)
       pw_point(sUV + (i & 1) * Dm::UVBUF, sJ + (i & 1) * 10, sJS + (i & 1) * Dm::JSBUF, zone_of(i));
+    if (PWG) {   // zone i's points are done: issue zone i+2 (its XE and R slots were last read for zone i)
+      cp_async_wait<0>();
+      pw_issue(i + 2);
+      pw_load_id(i + 3);
+      cp_async_commit();
+    }
     t_work += clock64() - t0;
     __syncthreads();
   }
+  if (PWG) cp_async_wait<0>();
   if (a.prof != nullptr && tid == 0) {
     a.prof[blockIdx.x * 16 + 0] = t_work;
     a.prof[blockIdx.x * 16 + 2] = clock64() - t_all;

@@ -42,7 +42,8 @@ struct V5Dims {
   static constexpr int OFF_RED = OFF_J + 20;
   static constexpr int OFF_ID = OFF_RED + 32;          // zone -> node ids of the next two zones, int32 [2][P^3]
   static constexpr int OFF_MB = OFF_ID + (2 * P3 + 1) / 2;   // two mbarriers (kb1_v10.cuh bulk copies)
-  static constexpr int TOTAL = OFF_MB + 2;
+  static constexpr int OFF_XEB = OFF_MB + 2;                  // second XE buffer (kb1_v10.cuh PWG)
+  static constexpr int TOTAL = OFF_XEB + XE;
   static constexpr int MT = (N + 7) / 8, KS_P = (P + 3) / 4, KS_N = (N + 3) / 4, KS_T = (T + 3) / 4;
 };
 
