@@ -219,6 +219,7 @@ KB1Variant select_variant(int dim, int k) {
       if (strcmp(force, "v10.q") == 0) { d = variant3v10<4, 0, 0, 4>(); d.name = "v10.q"; return d; }
       if (strcmp(force, "v10.b") == 0) { d = variant3v10<4, 0, 0, 1>(); d.name = "v10.b"; return d; }
       if (strcmp(force, "v10.l") == 0) { d = variant3v10<4, 0, 0, 2>(); d.name = "v10.l"; return d; }
+      if (strcmp(force, "v10.w16") == 0) { d = variant3v10<4, 0, 0, 16, 3>(); d.name = "v10.w16"; return d; }
       if (strcmp(force, "v10.x") == 0) { d = variant3v10<4, 0, 0, 8, 3>(); d.name = "v10.x"; return d; }
       if (strcmp(force, "v10.xd1") == 0) { d = variant3v10<4, 1, 0, 8, 3>(); d.name = "v10.xd1"; return d; }
       if (strcmp(force, "v10.xd2") == 0) { d = variant3v10<4, 2, 0, 8, 3>(); d.name = "v10.xd2"; return d; }

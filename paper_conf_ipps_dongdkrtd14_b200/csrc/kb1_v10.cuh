@@ -15,6 +15,7 @@
 // OPT bit 1 (LATE): the gather of zone i+1 is issued after the C^T stage of zone i-1 instead of before it,
 // away from the point warps' stage-C shared-memory burst at the start of every zone.
 // OPT bit 2 (BAL): forward stage B's 32 e items go two each to the 16 threads without a field item.
+// OPT bit 4 (V16): e and rho0|J0| (contiguous per zone) by 16-byte cp.async.
 // OPT bit 3 (PWG): the POINT warps issue the gather of zone i+2 at the end of their zone i (they finish
 // before the contraction warps, which are the bound), into a second XE buffer; completion reaches the
 // contraction warps through cp.async.mbarrier.arrive on a per-buffer mbarrier, so the contraction warps
@@ -34,6 +35,9 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned by
                    smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar))
                : "memory");
 }
+__device__ __forceinline__ void cp_async16(void *dst, const void *src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
 __device__ __forceinline__ void cp_async_mbar_arrive(uint64_t *bar) {
   asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(bar)) : "memory");
 }
@@ -48,7 +52,9 @@ template <int K, int DIAG = 0, int MODE = 0, int OPT = 0, int VMODE = 0>
 __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB1Args a) {
   using Dm = V5Dims<K>;
   using Cfg = KB1V5Cfg<K, MODE>;
-  constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4, PWG = OPT & 8;
+  constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4, PWG = OPT & 8, V16 = OPT & 16;
+  static_assert(!V16 || (Dm::T3 % 2 == 0 && Dm::N3 % 2 == 0 && Dm::XE_E % 2 == 0 && (Dm::OFF_XE + Dm::XE_E) % 2 == 0 &&
+                         (Dm::OFF_UV + Dm::O_R) % 2 == 0 && Dm::UVBUF % 2 == 0), "16-byte copies need 16-byte alignment");
   static_assert(!(PWG && (BULK || LATE)), "PWG replaces the contraction warps' gather");
   static_assert(!BULK || ((Dm::OFF_XE + Dm::XE_E) % 2 == 0 && (Dm::OFF_UV + Dm::O_R) % 2 == 0 && Dm::UVBUF % 2 == 0 &&
                           (Dm::T3 * 8) % 16 == 0 && (Dm::N3 * 8) % 16 == 0),
@@ -123,6 +129,10 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
           bulk_g2s(R, a.rho0detJ0 + z * N3, N3 * 8, bar);
         }
         if (ktid < 10) cp_async8(sXE + Dm::XE_J + ktid, ktid < 9 ? a.J0inv + z * 9 + ktid : a.zone_gamma + z, true);
+      } else if (V16) {   // e and rho0|J0| are contiguous per zone: 16-byte copies, half the instructions
+        for (int r = 2 * ktid; r < T3; r += 2 * NKW) cp_async16(sXE + Dm::XE_E + r, a.e + z * T3 + r);
+        if (ktid < 10) cp_async8(sXE + Dm::XE_J + ktid, ktid < 9 ? a.J0inv + z * 9 + ktid : a.zone_gamma + z, true);
+        for (int r = 2 * ktid; r < N3; r += 2 * NKW) cp_async16(R + r, a.rho0detJ0 + z * N3 + r);
       } else {
         for (int r = ktid; r < T3 + 10; r += NKW) {
           const double *src = r < T3 ? a.e + z * T3 + r : r < T3 + 9 ? a.J0inv + z * 9 + (r - T3) : a.zone_gamma + z;
