@@ -291,13 +291,16 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       constexpr int NTL = (N2 + 7) / 8;
       for (int tl = kwarp; tl < NTL; tl += NKWW) {
         const int colb = min(tl * 8 + lr, N2 - 1);
+        int soff[KS_N];   // swizzled slot of this lane's q0 = 4 s + lc in row colb (kb1_v6.cuh js_idx), once per tile
+#pragma unroll
+        for (int s = 0; s < KS_N; ++s) soff[s] = js_idx(colb, min(4 * s + lc, N - 1));
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           double sv[5][KS_N];
 #pragma unroll
           for (int c5 = 0; c5 < 5; ++c5)
 #pragma unroll
-            for (int s = 0; s < KS_N; ++s) sv[c5][s] = sb[(h * 5 + c5) * N3 + js_idx(colb, min(4 * s + lc, N - 1))];   // swizzled S (kb1_v6.cuh)
+            for (int s = 0; s < KS_N; ++s) sv[c5][s] = sb[(h * 5 + c5) * N3 + soff[s]];
           double d[5][2];
 #pragma unroll
           for (int c5 = 0; c5 < 5; ++c5) {

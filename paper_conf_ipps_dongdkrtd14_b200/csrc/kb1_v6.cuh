@@ -16,14 +16,20 @@
 // constant-bank operands with compile-time indices (kb1_v2.cuh's CT<K>), so a contraction stage is
 // LDS -> DFMA c[][] -> STS with no table loads.
 //
-// JS layout: J/S of point (col = q2*N + q1, q0) at col*8 + 2*((q0/2) ^ ((col/2) & 3)) + (q0 & 1): the
+// JS layout: J/S of point (col = q2*N + q1, q0) at col*8 + 2*((q0/2) ^ g(col)) + (q0 & 1) (js_idx): the
 // pair swizzle makes the contraction warps' 16-byte row accesses (8 consecutive cols, one q0 pair) and
 // the point warps' 8-byte accesses (4 q0 x 8 q1 per warp) both conflict-free.
 #pragma once
 #include "kb1_v5.cuh"
 
+// Pair slot of q0 in row col: (q0/2) ^ g(col), g = the 2-bit reversal of (col/2) & 3.  g is a bijection, so the
+// contraction warps' 16-byte row accesses (8 consecutive rows, one pair) stay conflict-free, and
+// g(1) ^ g(0) = g(3) ^ g(2) = 2, so the 8-byte accesses of a half-warp (rows c..c+3 of one slab x 4 q0: the
+// point warps and the DMMA fragments of kb1_v10.cuh) fill 16 distinct banks.  (The first form, (q0/2) ^
+// (col/2), left those 2-way conflicted: ncu on v10, profiles/r01_kw_stage_clocks.txt.)
 __device__ __forceinline__ int js_idx(int col, int q0) {
-  return col * 8 + ((((q0 >> 1) ^ (col >> 1)) & 3) << 1) + (q0 & 1);
+  const int g = (col & 2) | ((col >> 2) & 1);   // 2-bit reversal of (col / 2) & 3
+  return col * 8 + ((((q0 >> 1) ^ g) & 3) << 1) + (q0 & 1);
 }
 __device__ __forceinline__ void lds_f64x2(const double *src, double &a, double &b) {
   const unsigned s = (unsigned)__cvta_generic_to_shared(src);
