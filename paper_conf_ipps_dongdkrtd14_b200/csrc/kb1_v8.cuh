@@ -26,7 +26,10 @@ struct V8Dims {
   static constexpr int P2 = P * P, NK = P * P * P, NT = T * T * T, NS = N * N, T2 = T * T;
   static constexpr int PP = (P + 1) / 2 * 2;           // U row stride (16-byte pairs)
   static constexpr int SR = N + 2;                     // S row stride (conflict-free 16-byte row loads)
-  static constexpr int TAB = (2 * N * P + N * T + N + 1) / 2 * 2;
+  // Phi rows padded to TS = T + 1 doubles in shared memory: the point stage reads Phi[q0][j] with q0 per lane,
+  // and a row stride of T = 8 doubles put 16 lanes on 2 sixteen-byte slots (8-way; ncu on C5)
+  static constexpr int TS = T + 1;
+  static constexpr int TAB = (2 * N * P + N * TS + N + 1) / 2 * 2;
   static constexpr int O_X = 0, O_E = 6 * NK, O_AF = O_E + NT, O_AE = O_AF + 3 * NK, O_J0 = O_AE + NT;
   static constexpr int FIX = (O_J0 + 10 + 1) / 2 * 2;
   // region A: T (TB, TG [6][P2] each, TE [T2]) -> S [10][N][SR] -> Z (ZB, ZG [3][P2] each, ZE [T2])
@@ -58,7 +61,7 @@ __global__ void __launch_bounds__(KB1V8Cfg<K>::NTH, MINB) kb1_v8_3d(const KB1Arg
   static_assert(NTH >= 6 * 3 * P + T, "stage B: one item per thread");
   static_assert(NTH >= 3 * P2, "stage A^T: one item per thread");
   extern __shared__ double smem[];
-  double *sB = smem, *sG = sB + N * P, *sPhi = sG + N * P, *sW = sPhi + N * T;
+  double *sB = smem, *sG = sB + N * P, *sPhi = sG + N * P, *sW = sPhi + N * Dm::TS;
   double *sF = smem + Dm::OFF_FIX;
   double *sX = sF + Dm::O_X, *sE = sF + Dm::O_E, *sAF = sF + Dm::O_AF, *sAE = sF + Dm::O_AE, *sJ0 = sF + Dm::O_J0;
   double *sA = smem + Dm::OFF_A, *sBr = smem + Dm::OFF_B, *sRed = smem + Dm::OFF_RED;
@@ -68,7 +71,12 @@ __global__ void __launch_bounds__(KB1V8Cfg<K>::NTH, MINB) kb1_v8_3d(const KB1Arg
   const int64_t nn = a.num_nodes;
 
   // ---- a0: tables + gather ----------------------------------------------------------------------
-  for (int i = tid; i < 2 * N * P + N * T + N; i += NTH) smem[i] = __ldg(a.tab + i);
+  for (int i = tid; i < 2 * N * P + N * T + N; i += NTH) {   // B, G; Phi into rows of TS; W
+    const double t = __ldg(a.tab + i);
+    if (i < 2 * N * P) smem[i] = t;
+    else if (i < 2 * N * P + N * T) sPhi[((i - 2 * N * P) / T) * Dm::TS + (i - 2 * N * P) % T] = t;
+    else sW[i - 2 * N * P - N * T] = t;
+  }
   for (int r = tid; r < NK; r += NTH) {
     const int64_t node = __ldg(a.zone_nodes + z * NK + r);
 #pragma unroll
@@ -195,7 +203,7 @@ __global__ void __launch_bounds__(KB1V8Cfg<K>::NTH, MINB) kb1_v8_3d(const KB1Arg
       }
       double eq = 0.0;
 #pragma unroll
-      for (int j0 = 0; j0 < T; ++j0) eq = fma(sPhi[q0 * T + j0], sBr[18 * N * PP + q1 * T + j0], eq);
+      for (int j0 = 0; j0 < T; ++j0) eq = fma(sPhi[q0 * Dm::TS + j0], sBr[18 * N * PP + q1 * T + j0], eq);
       double Jm[3][3], Gv[3][3];
 #pragma unroll
       for (int c = 0; c < 3; ++c)
