@@ -176,7 +176,7 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
   if (dim == 3) {
     switch (k) {
       case 1: add(variant3v2<1, 32, 2, 1>(), "v2.p1.z32"); add(variant3v2<1, 64, 2>(), "v2.z64"); add(variant3<1, 32, 2>(), "v1.z32"); break;
-      case 2: add(variant3v2<2, 4, 3>(), "v2.z4"); add(variant3v2<2, 4, 2, 1>(), "v2.p1.z4"); add(variant3v2<2, 2, 4, 1>(), "v2.p1.z2"); add(variant3v3<2, 4, 2>(), "v3.z4"); add(variant3<2, 16, 2>(), "v1.z16"); break;
+      case 2: add(variant3v2<2, 1, 12>(), "v2.z1m12"); add(variant3v2<2, 2, 6>(), "v2.z2m6"); add(variant3v2<2, 4, 3>(), "v2.z4"); add(variant3v2<2, 4, 2, 1>(), "v2.p1.z4"); add(variant3v2<2, 2, 4, 1>(), "v2.p1.z2"); add(variant3v3<2, 4, 2>(), "v3.z4"); add(variant3<2, 16, 2>(), "v1.z16"); break;
       case 3: add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3v2<3, 1, 2, 1>(), "v2.p1.z1"); add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
       case 4:
         add(variant3v10<4, 0, 0, 0, 3>(), "v10.w"); add(variant3v10<4, 0, 0, 0, 2>(), "v10.v"); add(variant3v10<4>(), "v10"); add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
