@@ -24,6 +24,7 @@
 #include "kb1_v6.cuh"
 #include "kb1_v10.cuh"
 #include "kb1_v8.cuh"
+#include "kb1_p2d.cuh"
 #include "kb2_gather.cuh"
 #include "tables.h"
 #include "exchange.cuh"
@@ -162,6 +163,17 @@ KB1Variant variant3() {
                     (const void *)&kb1_corner_force_3d<K, ZPC, MINB>, false, nullptr};
 }
 template <int K, int ZPC, int MINB>
+void launchP2d(const KB1Args &a, int grid, cudaStream_t s) {
+  using C = KB1CfgP2d<K, ZPC>;
+  kb1_p2d<K, ZPC, MINB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+}
+template <int K, int ZPC, int MINB>
+KB1Variant variantP2d() {
+  using C = KB1CfgP2d<K, ZPC>;
+  return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launchP2d<K, ZPC, MINB>, (const void *)&kb1_p2d<K, ZPC, MINB>, true,
+                    nullptr};
+}
+template <int K, int ZPC, int MINB>
 KB1Variant variant2() {
   using C = KB1Cfg2<K, ZPC>;
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch2<K, ZPC, MINB>,
@@ -192,7 +204,7 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
       case 1: add(variant2<1, 64, 2>(), "v1-2d.z64"); break;
       case 2: add(variant2<2, 16, 2>(), "v1-2d.z16"); break;
       case 3: add(variant2<3, 8, 2>(), "v1-2d.z8"); break;
-      case 4: add(variant2<4, 4, 3>(), "v1-2d.z4m3"); add(variant2<4, 4, 2>(), "v1-2d.z4"); add(variant2<4, 2, 4>(), "v1-2d.z2m4"); break;
+      case 4: add(variantP2d<4, 2, 6>(), "p2d.z2m6"); add(variantP2d<4, 4, 3>(), "p2d.z4m3"); add(variant2<4, 4, 3>(), "v1-2d.z4m3"); add(variant2<4, 4, 2>(), "v1-2d.z4"); break;
       case 5: add(variant2<5, 2, 2>(), "v1-2d.z2"); break;
       case 6: add(variant2<6, 2, 2>(), "v1-2d.z2"); break;
       case 7: add(variant2<7, 1, 2>(), "v1-2d.z1"); break;
@@ -223,6 +235,7 @@ KB1Variant select_variant(int dim, int k) {
       if (strcmp(force, "v10.x") == 0) { d = variant3v10<4, 0, 0, 8, 3>(); d.name = "v10.x"; return d; }
       if (strcmp(force, "v10.xd1") == 0) { d = variant3v10<4, 1, 0, 8, 3>(); d.name = "v10.xd1"; return d; }
       if (strcmp(force, "v10.xd2") == 0) { d = variant3v10<4, 2, 0, 8, 3>(); d.name = "v10.xd2"; return d; }
+      if (strcmp(force, "v10.wr4") == 0) { d = variant3v10<4, 0, 4, 0, 3>(); d.name = "v10.wr4"; return d; }
       if (strcmp(force, "v10.wr3") == 0) { d = variant3v10<4, 0, 3, 0, 3>(); d.name = "v10.wr3"; return d; }
       if (strcmp(force, "v10.wd1") == 0) { d = variant3v10<4, 1, 0, 0, 3>(); d.name = "v10.wd1"; return d; }
       if (strcmp(force, "v10.vd1") == 0) { d = variant3v10<4, 1, 0, 0, 2>(); d.name = "v10.vd1"; return d; }

@@ -48,16 +48,16 @@ struct V5Dims {
 };
 
 // MODE picks the register split between the point warps and the DMMA warps (setmaxnreg) and the DMMA
-// tiles in flight per warp: 0 = 168 / 88 / 8, 1 = 184 / 72 / 4, 2 = 200 / 56 / 2, 3 = 176 / 80 / 4.
+// tiles in flight per warp: 0 = 168 / 88 / 8, 1 = 184 / 72 / 4, 2 = 200 / 56 / 2, 3 = 176 / 80 / 4, 4 = 160 / 96 / 8.
 template <int K, int MODE = 0>
 struct KB1V5Cfg {
   using Dm = V5Dims<K>;
   static constexpr int NPW = (Dm::N3 / 2 + 127) / 128 * 128;   // 2 points per point-thread
   static constexpr int NKW = 256;
   static constexpr int NTH = NPW + NKW;
-  static constexpr int REG_PW = MODE == 0 ? 168 : MODE == 1 ? 184 : MODE == 2 ? 200 : 176;
-  static constexpr int REG_KW = MODE == 0 ? 88 : MODE == 1 ? 72 : MODE == 2 ? 56 : 80;
-  static constexpr int KWCH = MODE == 0 ? 8 : MODE == 1 ? 4 : MODE == 2 ? 2 : 4;   // DMMA tiles in flight per warp
+  static constexpr int REG_PW = MODE == 0 ? 168 : MODE == 1 ? 184 : MODE == 2 ? 200 : MODE == 3 ? 176 : 160;
+  static constexpr int REG_KW = MODE == 0 ? 88 : MODE == 1 ? 72 : MODE == 2 ? 56 : MODE == 3 ? 80 : 96;
+  static constexpr int KWCH = MODE == 0 ? 8 : MODE == 1 ? 4 : MODE == 2 ? 2 : MODE == 3 ? 4 : 8;   // DMMA tiles in flight per warp
   static constexpr int REG_LAUNCH = (65536 / NTH) / 8 * 8;
   static_assert(NPW * REG_PW + NKW * REG_KW <= NTH * REG_LAUNCH, "register split exceeds the CTA's allocation");
   static constexpr int SMEM_BYTES = Dm::TOTAL * 8;

@@ -257,7 +257,7 @@ def test_every_kernel_variant(orc, k, name, monkeypatch):
     assert h.variant == name
 
 
-@pytest.mark.parametrize("name", ["v1-2d.z4m3", "v1-2d.z4", "v1-2d.z2m4"])
+@pytest.mark.parametrize("name", ["p2d.z2m6", "p2d.z4m3", "v1-2d.z4m3", "v1-2d.z4"])
 def test_every_2d_kernel_variant(orc, name, monkeypatch):
     """The 2D Q4 candidates (C2's order) meet the parity bar, on a mesh with a partial last zone batch."""
     monkeypatch.setenv("BLAST_CF_KB1", name)
