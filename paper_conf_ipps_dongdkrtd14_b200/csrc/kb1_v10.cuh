@@ -53,6 +53,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   using Dm = V5Dims<K>;
   using Cfg = KB1V5Cfg<K, MODE>;
   constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4, PWG = OPT & 8, V16 = OPT & 16;
+  constexpr bool NOXV = OPT & 32;   // timing diagnostic only (wrong results): no x / v gather
   static_assert(!V16 || (Dm::T3 % 2 == 0 && Dm::N3 % 2 == 0 && Dm::XE_E % 2 == 0 && (Dm::OFF_XE + Dm::XE_E) % 2 == 0 &&
                          (Dm::OFF_UV + Dm::O_R) % 2 == 0 && Dm::UVBUF % 2 == 0), "16-byte copies need 16-byte alignment");
   static_assert(!(PWG && (BULK || LATE)), "PWG replaces the contraction warps' gather");
@@ -112,7 +113,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   auto kw_issue = [&](int64_t i) {       // cp.async gather of zone i into XE and R of UV[i & 1]
     if (i < nz) {
       const int64_t z = zone_of(i);
-      if (ktid < P3) {
+      if (!NOXV && ktid < P3) {
         const int64_t node = sID[(i & 1) * P3 + ktid];
 #pragma unroll
         for (int c = 0; c < 3; ++c) {
