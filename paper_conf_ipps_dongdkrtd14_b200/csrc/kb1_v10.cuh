@@ -16,6 +16,7 @@
 // away from the point warps' stage-C shared-memory burst at the start of every zone.
 // OPT bit 2 (BAL): forward stage B's 32 e items go two each to the 16 threads without a field item.
 // OPT bit 4 (V16): e and rho0|J0| (contiguous per zone) by 16-byte cp.async.
+// OPT bit 6 (SPREAD): the x / v node gather spread over all contraction threads (3 copies each).
 // OPT bit 3 (PWG): the POINT warps issue the gather of zone i+2 at the end of their zone i (they finish
 // before the contraction warps, which are the bound), into a second XE buffer; completion reaches the
 // contraction warps through cp.async.mbarrier.arrive on a per-buffer mbarrier, so the contraction warps
@@ -54,6 +55,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   using Cfg = KB1V5Cfg<K, MODE>;
   constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4, PWG = OPT & 8, V16 = OPT & 16;
   constexpr bool NOXV = OPT & 32;   // timing diagnostic only (wrong results): no x / v gather
+  constexpr bool SPREAD = OPT & 64;   // the 6 P^3 node-field copies spread over all contraction threads
   static_assert(!V16 || (Dm::T3 % 2 == 0 && Dm::N3 % 2 == 0 && Dm::XE_E % 2 == 0 && (Dm::OFF_XE + Dm::XE_E) % 2 == 0 &&
                          (Dm::OFF_UV + Dm::O_R) % 2 == 0 && Dm::UVBUF % 2 == 0), "16-byte copies need 16-byte alignment");
   static_assert(!(PWG && (BULK || LATE)), "PWG replaces the contraction warps' gather");
@@ -113,7 +115,13 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   auto kw_issue = [&](int64_t i) {       // cp.async gather of zone i into XE and R of UV[i & 1]
     if (i < nz) {
       const int64_t z = zone_of(i);
-      if (!NOXV && ktid < P3) {
+      if (SPREAD) {   // item (f, a): warps 0-7 each take ~3 copies instead of warps 0-3 taking 6
+        for (int it2 = ktid; it2 < 6 * P3; it2 += NKW) {
+          const int f = it2 / P3, aa = it2 - f * P3;
+          const int64_t node = sID[(i & 1) * P3 + aa];
+          cp_async8(sXE + Dm::XE_X + f * P3 + aa, (f < 3 ? a.x + f * nn : a.v + (f - 3) * nn) + node, true);
+        }
+      } else if (!NOXV && ktid < P3) {
         const int64_t node = sID[(i & 1) * P3 + ktid];
 #pragma unroll
         for (int c = 0; c < 3; ++c) {
