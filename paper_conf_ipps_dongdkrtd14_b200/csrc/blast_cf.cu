@@ -235,6 +235,8 @@ KB1Variant select_variant(int dim, int k) {
       if (strcmp(force, "v10.x") == 0) { d = variant3v10<4, 0, 0, 8, 3>(); d.name = "v10.x"; return d; }
       if (strcmp(force, "v10.xd1") == 0) { d = variant3v10<4, 1, 0, 8, 3>(); d.name = "v10.xd1"; return d; }
       if (strcmp(force, "v10.xd2") == 0) { d = variant3v10<4, 2, 0, 8, 3>(); d.name = "v10.xd2"; return d; }
+      if (strcmp(force, "v10.wq") == 0) { d = variant3v10<4, 0, 0, 4, 3>(); d.name = "v10.wq"; return d; }
+      if (strcmp(force, "v10.wl") == 0) { d = variant3v10<4, 0, 0, 2, 3>(); d.name = "v10.wl"; return d; }
       if (strcmp(force, "v10.ws") == 0) { d = variant3v10<4, 0, 0, 64, 3>(); d.name = "v10.ws"; return d; }
       if (strcmp(force, "v10.wnoxv") == 0) { d = variant3v10<4, 0, 0, 32, 3>(); d.name = "v10.wnoxv"; return d; }
       if (strcmp(force, "v10.wr4") == 0) { d = variant3v10<4, 0, 4, 0, 3>(); d.name = "v10.wr4"; return d; }
