@@ -138,12 +138,12 @@ KB1Variant variant3v6() {
 template <int K, int DIAG, int MODE, int OPT, int VMODE>
 void launch3v10(const KB1Args &a, int grid, cudaStream_t s) {
   using C = KB1V5Cfg<K, MODE>;
-  kb1_v10_3d<K, DIAG, MODE, OPT, VMODE><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+  kb1_v10_3d<K, DIAG, MODE, OPT, VMODE><<<grid, C::NTH, v10_smem_bytes<K, OPT>(), s>>>(a);
 }
 template <int K, int DIAG = 0, int MODE = 0, int OPT = 0, int VMODE = 0>
 KB1Variant variant3v10() {
   using C = KB1V5Cfg<K, MODE>;
-  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v10<K, DIAG, MODE, OPT, VMODE>,
+  return KB1Variant{1, C::NTH, v10_smem_bytes<K, OPT>(), &launch3v10<K, DIAG, MODE, OPT, VMODE>,
                     (const void *)&kb1_v10_3d<K, DIAG, MODE, OPT, VMODE>, true, nullptr};
 }
 template <int K, int MINB>
@@ -191,7 +191,7 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
       case 2: add(variant3v2<2, 1, 12>(), "v2.z1m12"); add(variant3v2<2, 2, 6>(), "v2.z2m6"); add(variant3v2<2, 4, 3>(), "v2.z4"); add(variant3v2<2, 4, 2, 1>(), "v2.p1.z4"); add(variant3v2<2, 2, 4, 1>(), "v2.p1.z2"); add(variant3v3<2, 4, 2>(), "v3.z4"); add(variant3<2, 16, 2>(), "v1.z16"); break;
       case 3: add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3v2<3, 1, 2, 1>(), "v2.p1.z1"); add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
       case 4:
-        add(variant3v10<4, 0, 0, 0, 3>(), "v10.w"); add(variant3v10<4, 0, 0, 0, 2>(), "v10.v"); add(variant3v10<4>(), "v10"); add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
+        add(variant3v10<4, 0, 0, 0, 3>(), "v10.w"); add(variant3v10<4, 0, 0, 128, 3>(), "v10.wu"); add(variant3v10<4, 0, 0, 0, 2>(), "v10.v"); add(variant3v10<4>(), "v10"); add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
@@ -237,6 +237,8 @@ KB1Variant select_variant(int dim, int k) {
       if (strcmp(force, "v10.xd2") == 0) { d = variant3v10<4, 2, 0, 8, 3>(); d.name = "v10.xd2"; return d; }
       if (strcmp(force, "v10.wq") == 0) { d = variant3v10<4, 0, 0, 4, 3>(); d.name = "v10.wq"; return d; }
       if (strcmp(force, "v10.wl") == 0) { d = variant3v10<4, 0, 0, 2, 3>(); d.name = "v10.wl"; return d; }
+      if (strcmp(force, "v10.we") == 0) { d = variant3v10<4, 0, 0, 512, 3>(); d.name = "v10.we"; return d; }
+      if (strcmp(force, "v10.wpad") == 0) { d = variant3v10<4, 0, 0, 1024, 3>(); d.name = "v10.wpad"; return d; }
       if (strcmp(force, "v10.ws") == 0) { d = variant3v10<4, 0, 0, 64, 3>(); d.name = "v10.ws"; return d; }
       if (strcmp(force, "v10.wnoxv") == 0) { d = variant3v10<4, 0, 0, 32, 3>(); d.name = "v10.wnoxv"; return d; }
       if (strcmp(force, "v10.wr4") == 0) { d = variant3v10<4, 0, 4, 0, 3>(); d.name = "v10.wr4"; return d; }

@@ -49,9 +49,43 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned parity) {
       : "memory");
 }
 
+// OPT bit 7 (PADU): padded U layouts for the forward stage B stores.  With the natural layout
+// U[cm][q2][q1][a0] (q2 stride N*P = 40) a half-warp of stage B (16 consecutive (q2, a0) items, one q1)
+// touches only 10 distinct 8-byte banks (40 = 8 mod 16): 2-way conflicts on all 24 stores per item, and the
+// e items' UE[q2][q1][j0] (q2 stride 32) are 4-way.  PADU uses q2 stride UQ = 53 (= 5 mod 16: a half-warp's
+// 16 items land on 16 banks) and q1 stride UQ1 = 6 (keeps stage C's half-warps -- q2 pair x 8 q1 at fixed a0
+// -- and the point warps' 8 q1 per warp conflict-free), and UE q2 stride N*T + 4 (bit 9, PADE, alone).
+// Bank model: tools/v10_stageB_bank_model.py (stage B 784 -> 400 wavefronts per zone, stage C unchanged).
+// Measured (profiles/r01_bench_c4_v10wu_*.jsonl): store conflicts 23.6 M -> 10.8 M per launch, but 2.7 %
+// SLOWER: the extra 22.5 KB push the CTA past the 196 KB shared-memory carveout, L1 shrinks, and the
+// point warps' spill reloads miss (3.3 M -> 7.6 M local sectors).  v10.wpad (v10.w + the same 22.5 KB
+// unused, OPT bit 10) is exactly as slow, so the conflicts themselves were off the critical path.
+template <int K, bool PADU, bool PADE = PADU>
+struct V10Dims : V5Dims<K> {
+  using B = V5Dims<K>;
+  using B::N, B::P, B::T, B::N2, B::N3, B::TAB, B::JSBUF, B::XE, B::P3, B::O_UX, B::YZREG;
+  static_assert(!PADU || K == 4, "PADU strides are chosen for k = 4 (N = 8, P = 5)");
+  static constexpr int UQ = PADU ? 53 : N * P, UQ1 = PADU ? 6 : P, UM = N * UQ, UQE = PADE ? N * T + 4 : N * T;
+  static constexpr int O_UE = 9 * UM, O_R = (O_UE + N * UQE + 1) / 2 * 2, UVBUF = (O_R + N3 + 1) / 2 * 2;
+  static constexpr int FWREG = O_UX + 9 * UM;
+  static constexpr int WREG = ((FWREG > YZREG ? FWREG : YZREG) + 1) / 2 * 2;
+  static constexpr int OFF_JS = TAB, OFF_UV = OFF_JS + 2 * JSBUF, OFF_XE = OFF_UV + 2 * UVBUF, OFF_W = OFF_XE + XE;
+  static constexpr int OFF_J = OFF_W + WREG;
+  static constexpr int OFF_RED = OFF_J + 20;
+  static constexpr int OFF_ID = OFF_RED + 32;
+  static constexpr int OFF_MB = OFF_ID + (2 * P3 + 1) / 2;
+  static constexpr int OFF_XEB = OFF_MB + 2;
+  static constexpr int TOTAL = OFF_XEB + XE;
+};
+template <int K, int OPT>
+constexpr int v10_smem_bytes() {   // OPT bit 10: PADU's extra 2872 doubles, unused (diagnostic: the L1 share)
+  return (V10Dims<K, (OPT & 128) != 0, (OPT & 640) != 0>::TOTAL + ((OPT & 1024) ? 2872 : 0)) * 8;
+}
+
 template <int K, int DIAG = 0, int MODE = 0, int OPT = 0, int VMODE = 0>
 __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB1Args a) {
-  using Dm = V5Dims<K>;
+  using Dm = V10Dims<K, (OPT & 128) != 0, (OPT & 640) != 0>;   // OPT bit 9 (PADE): the UE padding alone
+  constexpr int UQ = Dm::UQ, UQ1 = Dm::UQ1, UM = Dm::UM, UQE = Dm::UQE;
   using Cfg = KB1V5Cfg<K, MODE>;
   constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4, PWG = OPT & 8, V16 = OPT & 16;
   constexpr bool NOXV = OPT & 32;   // timing diagnostic only (wrong results): no x / v gather
@@ -219,7 +253,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
           tb[a1] = Tr[Dm::O_T + ((f * 2 + 0) * N + q2) * P2 + a1 * P + a0];
           tg[a1] = Tr[Dm::O_T + ((f * 2 + 1) * N + q2) * P2 + a1 * P + a0];
         }
-        double *U0 = (f < 3 ? UX + f * 3 * N2 * P : ub + (f - 3) * 3 * N2 * P) + q2 * N * P + a0;
+        double *U0 = (f < 3 ? UX + f * 3 * UM : ub + (f - 3) * 3 * UM) + q2 * UQ + a0;
 #pragma unroll
         for (int q1 = 0; q1 < N; ++q1) {
           double u0 = 0.0, u1 = 0.0, u2 = 0.0;
@@ -229,9 +263,9 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
             u1 = fma(C.G(q1, a1), tb[a1], u1);
             u2 = fma(C.B(q1, a1), tg[a1], u2);
           }
-          U0[q1 * P] = u0;
-          U0[N2 * P + q1 * P] = u1;
-          U0[2 * N2 * P + q1 * P] = u2;
+          U0[q1 * UQ1] = u0;
+          U0[UM + q1 * UQ1] = u1;
+          U0[2 * UM + q1 * UQ1] = u2;
         }
       } else {
         const int r2 = r - 6 * N * P, q2 = r2 / T, j0 = r2 - q2 * T;
@@ -243,7 +277,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
           double ue = 0.0;
 #pragma unroll
           for (int j1 = 0; j1 < T; ++j1) ue = fma(C.Phi(q1, j1), te[j1], ue);
-          ub[Dm::O_UE + (q2 * N + q1) * T + j0] = ue;
+          ub[Dm::O_UE + q2 * UQE + q1 * T + j0] = ue;
         }
       }
     }}}
@@ -260,7 +294,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       const int cm = r / N2, col = r - cm * N2;   // cm is warp-uniform (N2 = 64)
       double uv[P];
 #pragma unroll
-      for (int a0 = 0; a0 < P; ++a0) uv[a0] = UX[cm * N2 * P + col * P + a0];
+      for (int a0 = 0; a0 < P; ++a0) uv[a0] = UX[cm * UM + (col / N) * UQ + (col % N) * UQ1 + a0];
       double o[N];
       if (cm % 3 == 0) {
 #pragma unroll
@@ -481,7 +515,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       for (int f = 0; f < 3; ++f)
 #pragma unroll
         for (int m = 0; m < 3; ++m) {
-          const double u = ub[(((f * 3 + m) * N + q2) * N + q1) * P + a0];
+          const double u = ub[(f * 3 + m) * UM + q2 * UQ + q1 * UQ1 + a0];
           ga[f * 3 + m] = fma(m == 0 ? gga : ba, u, ga[f * 3 + m]);
           gb[f * 3 + m] = fma(m == 0 ? ggb : bb, u, gb[f * 3 + m]);
         }
@@ -489,7 +523,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     double ea = 0.0, eb = 0.0;
 #pragma unroll
     for (int j0 = 0; j0 < T; ++j0) {
-      const double ue = ub[Dm::O_UE + col * T + j0];
+      const double ue = ub[Dm::O_UE + q2 * UQE + q1 * T + j0];
       ea = fma(tPhi[q0a * T + j0], ue, ea);
       eb = fma(tPhi[(q0a + NH) * T + j0], ue, eb);
     }
