@@ -60,7 +60,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned parity) {
 // SLOWER: the extra 22.5 KB push the CTA past the 196 KB shared-memory carveout, L1 shrinks, and the
 // point warps' spill reloads miss (3.3 M -> 7.6 M local sectors).  v10.wpad (v10.w + the same 22.5 KB
 // unused, OPT bit 10) is exactly as slow, so the conflicts themselves were off the critical path.
-template <int K, bool PADU, bool PADE = PADU>
+template <int K, bool PADU, bool PADE = PADU, bool XEB = true>
 struct V10Dims : V5Dims<K> {
   using B = V5Dims<K>;
   using B::N, B::P, B::T, B::N2, B::N3, B::TAB, B::JSBUF, B::XE, B::P3, B::O_UX, B::YZREG;
@@ -75,16 +75,16 @@ struct V10Dims : V5Dims<K> {
   static constexpr int OFF_ID = OFF_RED + 32;
   static constexpr int OFF_MB = OFF_ID + (2 * P3 + 1) / 2;
   static constexpr int OFF_XEB = OFF_MB + 2;
-  static constexpr int TOTAL = OFF_XEB + XE;
+  static constexpr int TOTAL = OFF_XEB + (XEB ? XE : 0);   // the second XE buffer serves PWG only
 };
 template <int K, int OPT>
 constexpr int v10_smem_bytes() {   // OPT bit 10: PADU's extra 2872 doubles, unused (diagnostic: the L1 share)
-  return (V10Dims<K, (OPT & 128) != 0, (OPT & 640) != 0>::TOTAL + ((OPT & 1024) ? 2872 : 0)) * 8;
+  return (V10Dims<K, (OPT & 128) != 0, (OPT & 640) != 0, (OPT & 8) || !(OPT & 2048)>::TOTAL + ((OPT & 1024) ? 2872 : 0)) * 8;
 }
 
 template <int K, int DIAG = 0, int MODE = 0, int OPT = 0, int VMODE = 0>
 __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB1Args a) {
-  using Dm = V10Dims<K, (OPT & 128) != 0, (OPT & 640) != 0>;   // OPT bit 9 (PADE): the UE padding alone
+  using Dm = V10Dims<K, (OPT & 128) != 0, (OPT & 640) != 0, (OPT & 8) || !(OPT & 2048)>;   // bit 11: no XEB   // OPT bit 9 (PADE): the UE padding alone
   constexpr int UQ = Dm::UQ, UQ1 = Dm::UQ1, UM = Dm::UM, UQE = Dm::UQE;
   using Cfg = KB1V5Cfg<K, MODE>;
   constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4, PWG = OPT & 8, V16 = OPT & 16;
