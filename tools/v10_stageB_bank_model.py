@@ -45,25 +45,7 @@ def stageC(S,R,MS,CS):
                 else: addrs.append(None)
             if any(a is not None for a in addrs): tot+=wf(addrs)
     return tot
-b0=stageB(40,5,320,960); c0=stageC(40,5,320,960)
-print("current UX: B",b0,"C",c0, "ub B", stageB(40,5,320,960,False))
-res=[]
-for S in range(40,80):
-  for R in range(5,10):
-    if S<8*R-3: continue
-    MS=8*S; MS+= (0)
-    for mp in range(0,16):
-      for cp in range(0,16):
-        ms=MS+mp; cs=3*ms+cp
-        b=stageB(S,R,ms,cs); c=stageC(S,R,ms,cs)
-        res.append((b+c,b,c,S,R,mp,cp))
-res.sort(); print(res[:10])
 # ub alone
-r2=[]
-for S in range(40,80):
-  b=stageB(S,5,8*S,24*S,False); r2.append((b,S))
-r2.sort(); print("ub",r2[:5])
-print("ub S53 R6", stageB(53,6,424,3*424,False), "UX", stageB(53,6,424,1272), stageC(53,6,424,1272))
 def stageBe(SE):
     tot=0
     # e items r in 240..271 -> first 16 in blk0 (threads 240..255), 16 in blk1 threads 0..15 (non-BAL)
@@ -76,7 +58,6 @@ def stageBe(SE):
             addrs += [None]*(32-len(addrs))
             tot+=wf(addrs)
     return tot
-for SE in (32,36,40,44): print("UE",SE,stageBe(SE))
 def pw(S,R):
     tot=0
     for a0 in range(5):
@@ -85,4 +66,27 @@ def pw(S,R):
             q1=(l//4)%8; addrs.append(S*0+q1*R+a0)
         tot+=wf(addrs)
     return tot
-print("pw", pw(40,5), pw(53,6))
+
+
+if __name__ == "__main__":
+    b0=stageB(40,5,320,960); c0=stageC(40,5,320,960)
+    print("current UX: B",b0,"C",c0, "ub B", stageB(40,5,320,960,False))
+    res=[]
+    for S in range(40,80):
+      for R in range(5,10):
+        if S<8*R-3: continue
+        MS=8*S; MS+= (0)
+        for mp in range(0,16):
+          for cp in range(0,16):
+            ms=MS+mp; cs=3*ms+cp
+            b=stageB(S,R,ms,cs); c=stageC(S,R,ms,cs)
+            res.append((b+c,b,c,S,R,mp,cp))
+    res.sort(); print(res[:10])
+    r2=[]
+    for S in range(40,80):
+      b=stageB(S,5,8*S,24*S,False); r2.append((b,S))
+    r2.sort(); print("ub",r2[:5])
+    print("ub S53 R6", stageB(53,6,424,3*424,False), "UX", stageB(53,6,424,1272), stageC(53,6,424,1272))
+    for SE in (32,36,40,44): print("UE",SE,stageBe(SE))
+    print("pw", pw(40,5), pw(53,6))
+
