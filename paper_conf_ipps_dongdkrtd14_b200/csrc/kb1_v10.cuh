@@ -57,8 +57,8 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, unsigned parity) {
 // -- and the point warps' 8 q1 per warp conflict-free), and UE q2 stride N*T + 4 (bit 9, PADE, alone).
 // Bank model: tools/v10_stageB_bank_model.py (stage B 784 -> 400 wavefronts per zone, stage C unchanged).
 // Measured (profiles/r01_bench_c4_v10wu_*.jsonl): store conflicts 23.6 M -> 10.8 M per launch, but 2.7 %
-// SLOWER: the extra 22.5 KB push the CTA past the 196 KB shared-memory carveout, L1 shrinks, and the
-// point warps' spill reloads miss (3.3 M -> 7.6 M local sectors).  v10.wpad (v10.w + the same 22.5 KB
+// SLOWER: the extra 22.5 KB shrink L1 (228 KB - shared) from ~33 to ~10 KB, below the point warps' 30 KB
+// spill working set, and the spill reloads miss (3.3 M -> 7.6 M local sectors).  v10.wpad (v10.w + the same 22.5 KB
 // unused, OPT bit 10) is exactly as slow, so the conflicts themselves were off the critical path.
 template <int K, bool PADU, bool PADE = PADU, bool XEB = true>
 struct V10Dims : V5Dims<K> {
