@@ -238,6 +238,7 @@ KB1Variant select_variant(int dim, int k) {
       if (strcmp(force, "v10.wq") == 0) { d = variant3v10<4, 0, 0, 4, 3>(); d.name = "v10.wq"; return d; }
       if (strcmp(force, "v10.wl") == 0) { d = variant3v10<4, 0, 0, 2, 3>(); d.name = "v10.wl"; return d; }
       if (strcmp(force, "v10.we") == 0) { d = variant3v10<4, 0, 0, 512, 3>(); d.name = "v10.we"; return d; }
+      if (strcmp(force, "v10.wr1") == 0) { d = variant3v10<4, 0, 1, 0, 3>(); d.name = "v10.wr1"; return d; }
       if (strcmp(force, "v10.wn") == 0) { d = variant3v10<4, 0, 0, 2048, 3>(); d.name = "v10.wn"; return d; }
       if (strcmp(force, "v10.wpad") == 0) { d = variant3v10<4, 0, 0, 1024, 3>(); d.name = "v10.wpad"; return d; }
       if (strcmp(force, "v10.ws") == 0) { d = variant3v10<4, 0, 0, 64, 3>(); d.name = "v10.ws"; return d; }
