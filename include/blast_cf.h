@@ -38,7 +38,7 @@ extern "C" {
 enum {
   BLAST_CF_OK = 0,
   BLAST_CF_EINVAL = 1,       /* null / inconsistent argument */
-  BLAST_CF_EUNSUPPORTED = 2, /* dim/order outside {2,3} x [1,8], or non-affine initial zones with viscosity on */
+  BLAST_CF_EUNSUPPORTED = 2, /* dim/order outside {2,3} x [1,8] */
   BLAST_CF_ENOMEM = 3,       /* device or host allocation failed */
   BLAST_CF_ECUDA = 4,        /* CUDA runtime error (launch or asynchronous fault) */
   BLAST_CF_ENCCL = 5         /* NCCL error in the multi-GPU shared-DOF exchange */
@@ -88,6 +88,14 @@ void blast_cf_default_params(blast_cf_params *p);
  * nranks > 1 with nccl_unique_id NULL creates a "loopback" handle for blast_cf_eval_loopback (tests). */
 int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_cf_params *params,
                     void *cuda_stream, const void *nccl_unique_id, blast_cf **out);
+/* Initial geometry (reading R19).  The viscosity length scale l = h0 |J J0^{-1} s| needs J0^{-1} at every
+ * quadrature point; J varies inside a zone on curvilinear meshes (§2).  create
+ * checks whether every initial zone is affine (x0 = X0 + J0 xi at all its nodes, to 1e-11 relative):
+ *   affine      -> one J0^{-1} per zone ([Z][dim^2], 72 bytes/zone in 3D), the fast kernels;
+ *   non-affine  -> (viscosity on) J0^{-1} at every quadrature point ([Z][Nq][dim^2], computed once on the
+ *                  device from x0 by the same tensor-product basis gradients), evaluated by the generic
+ *                  per-slab kernels (the only candidates that read it); h0 then uses the quadrature volume
+ *                  sum_z sum_q alpha_q det J0(q). */
 
 /* One corner-force evaluation.  All seven arrays are DEVICE pointers owned by the caller:
  *   x, v        [dim][num_nodes]  current positions and velocities (SoA)
@@ -108,10 +116,18 @@ int blast_cf_eval(blast_cf *h, const double *x, const double *v, const double *e
  * staging buffers, two internal copy streams and the zone-chunk plan are created by the first call and
  * reused.  On large meshes the copies overlap the computation chunk by chunk (zones in contiguous
  * chunks; a chunk's corner force starts when its node prefix of x, v and its e, rho0detJ0 slices have
- * arrived); the results are bitwise those of blast_cf_eval on the same data.  Errors: EINVAL for NULL
- * arrays, ENOMEM / ECUDA as blast_cf_eval. */
+ * arrived); the results are bitwise those of blast_cf_eval on the same data.  rho0detJ0 NULL: use the
+ * copy made resident by blast_cf_set_rho0detJ0_host (no upload).  Errors: EINVAL for NULL arrays (or a
+ * NULL rho0detJ0 without a resident copy), ENOMEM / ECUDA as blast_cf_eval. */
 int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
                        double *out_Fdot1, double *out_FTv, double *out_dt_min);
+
+/* rho0 |J0| is time-invariant (strong mass conservation, reading R2), and the paper sends only the state
+ * (v, e, x) to the device each step (§3.1.2).  This copies rho0detJ0 (HOST
+ * [num_zones][Nq], pinned recommended) into the handle's staging buffer once (synchronous);
+ * blast_cf_eval_host(h, x, v, e, NULL, ...) then reads that resident copy instead of uploading one per
+ * call.  A later call replaces it.  EINVAL for NULL. */
+int blast_cf_set_rho0detJ0_host(blast_cf *h, const double *rho0detJ0);
 
 /* Tests only: the zone-local corner force matrices F_z = A_z B^T ([num_zones][dim*Nk][Nt], device), as
  * formed by kernel 7 of the paper.  Production eval never forms them. */

@@ -89,6 +89,7 @@ def lib():
                                   ctypes.POINTER(vp)]
     L.blast_cf_eval.argtypes = [vp] * 8
     L.blast_cf_eval_host.argtypes = [vp] * 8
+    L.blast_cf_set_rho0detJ0_host.argtypes = [vp, vp]
     L.blast_cf_eval_debug_Fz.argtypes = [vp] * 6
     L.blast_cf_get_info.argtypes = [vp, ctypes.POINTER(Info)]
     L.blast_cf_set_timing.argtypes = [vp, ctypes.c_int]
@@ -122,7 +123,7 @@ def lib():
     for f in ("blast_cf_rk2_create", "blast_cf_rk2_step", "blast_cf_rk2_rates", "blast_cf_rk2_mass_apply",
               "blast_cf_rk2_energy", "blast_cf_rk2_destroy", "blast_cf_rk2_advance", "blast_cf_rk2_setup_loopback",
               "blast_cf_rk2_rates_loopback", "blast_cf_rk2_energy_loopback",
-              "blast_cf_create", "blast_cf_eval", "blast_cf_eval_host", "blast_cf_eval_debug_Fz", "blast_cf_get_info",
+              "blast_cf_create", "blast_cf_eval", "blast_cf_eval_host", "blast_cf_set_rho0detJ0_host", "blast_cf_eval_debug_Fz", "blast_cf_get_info",
               "blast_cf_set_timing", "blast_cf_kernel_times", "blast_cf_destroy", "blast_cf_nccl_unique_id_size",
               "blast_cf_nccl_get_unique_id", "blast_cf_exchange_plan", "blast_cf_owner_mask", "blast_cf_debug_cta_dt",
               "blast_cf_debug_stage_clocks", "blast_cf_eval_loopback", "blast_cf_autotune"):
@@ -265,22 +266,46 @@ class CornerForce:
         return F1, FTv, dt
 
     def eval_host(self, x, v, e, rho0detJ0, out=None):
-        """Host-buffer evaluation (numpy arrays or pinned CPU tensors); synchronous."""
+        """Host-buffer evaluation (numpy arrays or pinned CPU tensors); synchronous.  rho0detJ0=None: use the
+        copy made resident by set_rho0detJ0_host (no upload per call)."""
         d, nn, Z = self.dim, self.num_nodes, self.num_zones
         if out is None:
             out = (np.empty((d, nn)), np.empty((Z, self.nt)), np.empty(1))
 
         def hp(a, shape):
+            # the C side reads / writes 8 bytes per element of HOST memory: float64, CPU, contiguous
             if hasattr(a, "data_ptr"):
-                assert a.dtype.is_floating_point and a.is_contiguous() and tuple(a.shape) == tuple(shape)
+                import torch
+                if not (a.dtype == torch.float64 and a.device.type == "cpu" and a.is_contiguous()
+                        and tuple(a.shape) == tuple(shape)):
+                    raise ValueError(f"eval_host needs contiguous float64 CPU tensors of shape {tuple(shape)}, got "
+                                     f"{a.dtype} on {a.device} with shape {tuple(a.shape)}")
                 return ctypes.c_void_p(a.data_ptr())
-            assert a.dtype == np.float64 and a.flags.c_contiguous and a.shape == tuple(shape)
+            if not (isinstance(a, np.ndarray) and a.dtype == np.float64 and a.flags.c_contiguous
+                    and a.shape == tuple(shape)):
+                raise ValueError(f"eval_host needs C-contiguous float64 arrays of shape {tuple(shape)}")
             return ctypes.c_void_p(a.ctypes.data)
 
         _check(lib().blast_cf_eval_host(self._h, hp(x, (d, nn)), hp(v, (d, nn)), hp(e, (Z, self.nt)),
-                                        hp(rho0detJ0, (Z, self.nq)), hp(out[0], (d, nn)), hp(out[1], (Z, self.nt)),
-                                        hp(out[2], (1,))), "blast_cf_eval_host")
+                                        None if rho0detJ0 is None else hp(rho0detJ0, (Z, self.nq)),
+                                        hp(out[0], (d, nn)), hp(out[1], (Z, self.nt)), hp(out[2], (1,))),
+               "blast_cf_eval_host")
         return out
+
+    def set_rho0detJ0_host(self, rho0detJ0):
+        """Make the time-invariant rho0|J0| (host array) resident for eval_host(..., rho0detJ0=None, ...)."""
+        a = rho0detJ0
+        shape = (self.num_zones, self.nq)
+        if hasattr(a, "data_ptr"):
+            import torch
+            if not (a.dtype == torch.float64 and a.device.type == "cpu" and a.is_contiguous() and tuple(a.shape) == shape):
+                raise ValueError(f"set_rho0detJ0_host needs a contiguous float64 CPU tensor of shape {shape}")
+            p = a.data_ptr()
+        else:
+            if not (isinstance(a, np.ndarray) and a.dtype == np.float64 and a.flags.c_contiguous and a.shape == shape):
+                raise ValueError(f"set_rho0detJ0_host needs a C-contiguous float64 array of shape {shape}")
+            p = a.ctypes.data
+        _check(lib().blast_cf_set_rho0detJ0_host(self._h, ctypes.c_void_p(p)), "blast_cf_set_rho0detJ0_host")
 
     def eval_debug_Fz(self, x, v, e, rho0detJ0):
         import torch

@@ -70,6 +70,7 @@ struct KB1Variant {
   const void *func;
   bool persistent;   // grid = resident CTAs; CTA c runs zone batches c, c + grid, ...
   const char *name = nullptr;
+  bool point_j0 = false;   // reads KB1Args::J0inv_q (per-point J0^{-1} of non-affine initial meshes)
 };
 
 template <int K, int ZPC, int MINB>
@@ -160,7 +161,7 @@ template <int K, int ZPC, int MINB>
 KB1Variant variant3() {
   using C = KB1Cfg3<K, ZPC>;
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3<K, ZPC, MINB>,
-                    (const void *)&kb1_corner_force_3d<K, ZPC, MINB>, false, nullptr};
+                    (const void *)&kb1_corner_force_3d<K, ZPC, MINB>, false, nullptr, true};
 }
 template <int K, int ZPC, int MINB>
 void launchP2d(const KB1Args &a, int grid, cudaStream_t s) {
@@ -177,7 +178,7 @@ template <int K, int ZPC, int MINB>
 KB1Variant variant2() {
   using C = KB1Cfg2<K, ZPC>;
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch2<K, ZPC, MINB>,
-                    (const void *)&kb1_corner_force_2d<K, ZPC, MINB>, false, nullptr};
+                    (const void *)&kb1_corner_force_2d<K, ZPC, MINB>, false, nullptr, true};
 }
 
 // Candidate KB1 variants per (dim, k), default first (f3 of SURVEY §8: the create-time default is the
@@ -188,10 +189,12 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
   if (dim == 3) {
     switch (k) {
       case 1: add(variant3v2<1, 32, 2, 1>(), "v2.p1.z32"); add(variant3v2<1, 64, 2>(), "v2.z64"); add(variant3<1, 32, 2>(), "v1.z32"); break;
-      case 2: add(variant3v2<2, 1, 12>(), "v2.z1m12"); add(variant3v2<2, 2, 6>(), "v2.z2m6"); add(variant3v2<2, 4, 3>(), "v2.z4"); add(variant3v2<2, 4, 2, 1>(), "v2.p1.z4"); add(variant3v2<2, 2, 4, 1>(), "v2.p1.z2"); add(variant3v3<2, 4, 2>(), "v3.z4"); add(variant3<2, 16, 2>(), "v1.z16"); break;
+      case 2: add(variant3v2<2, 1, 12>(), "v2.z1m12"); add(variant3v2<2, 2, 6>(), "v2.z2m6"); add(variant3v2<2, 2, 4, 1>(), "v2.p1.z2"); add(variant3<2, 16, 2>(), "v1.z16"); break;
       case 3: add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3v2<3, 1, 2, 1>(), "v2.p1.z1"); add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
       case 4:
-        add(variant3v10<4, 0, 0, 0, 3>(), "v10.w"); add(variant3v10<4, 0, 0, 128, 3>(), "v10.wu"); add(variant3v10<4, 0, 0, 0, 2>(), "v10.v"); add(variant3v10<4>(), "v10"); add(variant3v5<4, 0, 1>(), "v5.r1"); add(variant3v4<4, 0>(), "v4.m0"); add(variant3v5<4>(), "v5"); add(variant3v6<4>(), "v6"); add(variant3v4<4, 1>(), "v4.m1"); add(variant3v3<4, 1, 2>(), "v3.z1");
+        // (round 2: the superseded generations v10 (runtime switches), v10.wu, v6, v5, v4.m0/m1, v3.z1 that never
+        //  won the autotuner are no longer instantiated; DESIGN.md §10 keeps their measurements)
+        add(variant3v10<4, 0, 0, 0, 3>(), "v10.w"); add(variant3v10<4, 0, 0, 0, 2>(), "v10.v"); add(variant3v5<4, 0, 1>(), "v5.r1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
@@ -214,14 +217,24 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
   return v;
 }
 
-KB1Variant select_variant(int dim, int k) {
-  const std::vector<KB1Variant> c = kb1_candidates(dim, k);
+// the candidates a handle may use: all of them, or (non-affine initial mesh) those that read J0inv_q
+std::vector<KB1Variant> kb1_usable(int dim, int k, bool need_point_j0) {
+  std::vector<KB1Variant> c = kb1_candidates(dim, k);
+  if (need_point_j0) c.erase(std::remove_if(c.begin(), c.end(), [](const KB1Variant &x) { return !x.point_j0; }), c.end());
+  return c;
+}
+
+KB1Variant select_variant(int dim, int k, bool need_point_j0) {
+  const std::vector<KB1Variant> c = kb1_usable(dim, k, need_point_j0);
   if (c.empty()) return KB1Variant{0, 0, 0, nullptr, nullptr, false, nullptr};
   const char *force = getenv("BLAST_CF_KB1");   // experiments: pick a candidate by name
   if (force) {
     for (const KB1Variant &x : c)
       if (strcmp(x.name, force) == 0) return x;
-    // timing diagnostics (wrong results by design; never candidates of the autotuner)
+#ifdef BLAST_CF_DIAGNOSTICS
+    if (need_point_j0) return c[0];
+    // timing diagnostics (wrong results by design; never candidates of the autotuner): compiled only into a
+    // -DBLAST_CF_DIAGNOSTICS build, never into the production library
     if (dim == 3 && k == 4) {
       KB1Variant d;
       if (strcmp(force, "v5.d1") == 0) { d = variant3v5<4, 1>(); d.name = "v5.d1"; return d; }
@@ -253,6 +266,7 @@ KB1Variant select_variant(int dim, int k) {
       if (strcmp(force, "v5.r1d1") == 0) { d = variant3v5<4, 1, 1>(); d.name = "v5.r1d1"; return d; }
       if (strcmp(force, "v5.r2d1") == 0) { d = variant3v5<4, 1, 2>(); d.name = "v5.r2d1"; return d; }
     }
+#endif
   }
   return c[0];
 }
@@ -284,6 +298,59 @@ __global__ void kbd_form_Fz(const double *Sq, const double *tab, int k, int64_t 
       s += acc * phi;
     }
     Fz[(z * D * nk + row) * nt + j] = s;
+  }
+}
+
+// J0^{-1} at every quadrature point of a (non-affine) initial mesh, and alpha_q det J0(q) for its volume:
+// J0(q)_{cd} = sum_a x0_c(node_a) dW_a/dxi_d(q) with the tensor-product Lagrange tables of this order
+// (the a1 geometry step of SURVEY §8(a), on x0; reading R19).  One thread per (zone, point); dense over
+// the Nk nodes (a create-time cost, like the paper's per-run setup).
+template <int D>
+__global__ void kb0_point_j0inv(const double *x0, const int32_t *zn, const double *tab, int k, int64_t Z, int64_t nn,
+                                double *J0inv_q, double *wdet) {
+  const int n = 2 * k, p = k + 1;
+  const int nq = D == 3 ? n * n * n : n * n, nk = D == 3 ? p * p * p : p * p;
+  const double *B = tab, *G = tab + n * p, *w = tab + 2 * n * p + n * k;
+  const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= Z * nq) return;
+  const int64_t z = idx / nq;
+  const int q = (int)(idx - z * nq);
+  const int qi[3] = {q % n, (q / n) % n, q / (n * n)};
+  double J[D][D];
+  for (int c = 0; c < D; ++c)
+    for (int d = 0; d < D; ++d) J[c][d] = 0.0;
+  for (int a = 0; a < nk; ++a) {
+    const int ai[3] = {a % p, (a / p) % p, a / (p * p)};
+    const int64_t node = zn[z * nk + a];
+    double g[D];
+    for (int d = 0; d < D; ++d) {
+      double f = 1.0;
+      for (int t = 0; t < D; ++t) f *= (t == d ? G : B)[qi[t] * p + ai[t]];
+      g[d] = f;
+    }
+    for (int c = 0; c < D; ++c) {
+      const double xc = x0[c * nn + node];
+      for (int d = 0; d < D; ++d) J[c][d] = fma(xc, g[d], J[c][d]);
+    }
+  }
+  double alpha = 1.0;
+  for (int t = 0; t < D; ++t) alpha *= w[qi[t]];
+  double *o = J0inv_q + idx * D * D;
+  if (D == 2) {
+    const double det = J[0][0] * J[1][1] - J[0][1] * J[1][0], id = 1.0 / det;
+    o[0] = J[1][1] * id; o[1] = -J[0][1] * id; o[2] = -J[1][0] * id; o[3] = J[0][0] * id;
+    wdet[idx] = alpha * det;
+  } else {
+    const double c00 = J[1][1] * J[2][2] - J[1][2] * J[2][1], c01 = J[0][2] * J[2][1] - J[0][1] * J[2][2],
+                 c02 = J[0][1] * J[1][2] - J[0][2] * J[1][1], c10 = J[1][2] * J[2][0] - J[1][0] * J[2][2],
+                 c11 = J[0][0] * J[2][2] - J[0][2] * J[2][0], c12 = J[0][2] * J[1][0] - J[0][0] * J[1][2],
+                 c20 = J[1][0] * J[2][1] - J[1][1] * J[2][0], c21 = J[0][1] * J[2][0] - J[0][0] * J[2][1],
+                 c22 = J[0][0] * J[1][1] - J[0][1] * J[1][0];
+    const double det = J[0][0] * c00 + J[0][1] * c10 + J[0][2] * c20, id = 1.0 / det;
+    o[0] = c00 * id; o[1] = c01 * id; o[2] = c02 * id;
+    o[3] = c10 * id; o[4] = c11 * id; o[5] = c12 * id;
+    o[6] = c20 * id; o[7] = c21 * id; o[8] = c22 * id;
+    wdet[idx] = alpha * det;
   }
 }
 
@@ -424,6 +491,8 @@ struct blast_cf {
   int64_t ncta_cap = 0;
   // device memory
   double *d_tab = nullptr, *d_J0inv = nullptr, *d_gamma = nullptr, *d_Fz1 = nullptr, *d_ctadt = nullptr;
+  double *d_J0inv_q = nullptr;   // [Z][Nq][dim^2]: non-affine initial mesh with viscosity on (reading R19)
+  bool rho_resident = false;     // blast_cf_set_rho0detJ0_host has filled the staging copy of rho0|J0|
   int32_t *d_zone_nodes = nullptr, *d_ptr = nullptr, *d_ent = nullptr;
   // host-eval staging (blast_cf_eval_host): device copies of the inputs/outputs and the zone-chunk pipeline
   double *d_in = nullptr, *d_out = nullptr;
@@ -450,7 +519,7 @@ namespace {
 
 void free_handle(blast_cf *h) {
   if (!h) return;
-  cudaFree(h->d_tab); cudaFree(h->d_J0inv); cudaFree(h->d_gamma); cudaFree(h->d_Fz1); cudaFree(h->d_ctadt);
+  cudaFree(h->d_tab); cudaFree(h->d_J0inv); cudaFree(h->d_J0inv_q); cudaFree(h->d_gamma); cudaFree(h->d_Fz1); cudaFree(h->d_ctadt);
   cudaFree(h->d_zone_nodes); cudaFree(h->d_ptr); cudaFree(h->d_ent); cudaFree(h->d_in); cudaFree(h->d_out); cudaFree(h->d_prof);
   for (auto &e : h->ev)
     if (e) cudaEventDestroy(e);
@@ -633,10 +702,36 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
     for (int c = 0; c < dim; ++c)
       for (int d = 0; d < dim; ++d) J0inv[(size_t)z * dim * dim + c * dim + d] = (double)inv[c][d];
   }
-  if (!affine && h->params.use_viscosity)
-    return bail(fail(BLAST_CF_EUNSUPPORTED,
-                     "initial zone %lld is not affine: the viscosity length scale needs per-point J0 (not built)",
-                     (long long)bad_zone));
+  (void)bad_zone;
+  const bool point_j0 = !affine && h->params.use_viscosity;   // reading R19: J0^{-1} at every point
+  if (!affine) {   // the mesh volume by quadrature (the vertex-difference det above is exact only for affine zones)
+    const int64_t npts = Z * nq;
+    double *dx0 = nullptr, *dtab = nullptr, *dw = nullptr;
+    int32_t *dzn = nullptr;
+    std::vector<double> w((size_t)std::max<int64_t>(npts, 1));
+    int rc2 = BLAST_CF_OK;
+    if ((rc2 = upload(&dx0, mesh->x0, (size_t)dim * nn)) || (rc2 = upload(&dtab, tab.data(), tab.size())) ||
+        (rc2 = upload(&dzn, mesh->zone_nodes, (size_t)Z * nk))) {
+      cudaFree(dx0); cudaFree(dtab); cudaFree(dzn);
+      return bail(rc2);
+    }
+    if (cudaMalloc(&h->d_J0inv_q, std::max<int64_t>(npts, 1) * dim * dim * sizeof(double)) != cudaSuccess ||
+        cudaMalloc(&dw, std::max<int64_t>(npts, 1) * sizeof(double)) != cudaSuccess) {
+      cudaFree(dx0); cudaFree(dtab); cudaFree(dzn); cudaFree(dw);
+      return bail(fail(BLAST_CF_ENOMEM, "per-point J0 buffer (%lld points)", (long long)npts));
+    }
+    if (npts > 0) {
+      const unsigned blocks = (unsigned)((npts + 127) / 128);
+      if (dim == 3) kb0_point_j0inv<3><<<blocks, 128>>>(dx0, dzn, dtab, order, Z, nn, h->d_J0inv_q, dw);
+      else kb0_point_j0inv<2><<<blocks, 128>>>(dx0, dzn, dtab, order, Z, nn, h->d_J0inv_q, dw);
+    }
+    const cudaError_t ce = npts > 0 ? cudaMemcpy(w.data(), dw, npts * sizeof(double), cudaMemcpyDeviceToHost) : cudaSuccess;
+    cudaFree(dx0); cudaFree(dtab); cudaFree(dzn); cudaFree(dw);
+    if (ce != cudaSuccess) return bail(fail(BLAST_CF_ECUDA, "per-point J0 kernel: %s", cudaGetErrorString(ce)));
+    vol = 0.0L;
+    for (int64_t i = 0; i < npts; ++i) vol += (long double)w[i];
+    if (!point_j0) { cudaFree(h->d_J0inv_q); h->d_J0inv_q = nullptr; }
+  }
 
   // ---- multi-GPU: communicator, global volume / zone count for h0 ----
   double gvol = (double)vol, gz = (double)Z;
@@ -672,10 +767,10 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
   }
 
   // ---- kernel variant ----
-  h->var = select_variant(dim, order);
+  h->var = select_variant(dim, order, point_j0);
   if (!h->var.launch) return bail(fail(BLAST_CF_EUNSUPPORTED, "no kernel for dim %d order %d", dim, order));
   if ((rc = apply_variant(h, h->var))) return bail(rc);
-  for (const KB1Variant &c : kb1_candidates(dim, order))   // per-CTA dt slots for any candidate
+  for (const KB1Variant &c : kb1_usable(dim, order, point_j0))   // per-CTA dt slots for any candidate
     h->ncta_cap = std::max<int64_t>(h->ncta_cap, (Z + c.zpc - 1) / c.zpc);
 
   // ---- uploads ----
@@ -705,7 +800,7 @@ static int eval_impl(blast_cf *h, const double *x, const double *v, const double
   if (rc) return rc;
   KB1Args a;
   a.x = x; a.v = v; a.e = e; a.rho0detJ0 = rho0detJ0;
-  a.zone_nodes = h->d_zone_nodes; a.J0inv = h->d_J0inv; a.zone_gamma = h->d_gamma; a.tab = h->d_tab;
+  a.zone_nodes = h->d_zone_nodes; a.J0inv = h->d_J0inv; a.J0inv_q = h->d_J0inv_q; a.zone_gamma = h->d_gamma; a.tab = h->d_tab;
   a.Fz1 = h->d_Fz1; a.FTv = out_FTv; a.cta_dt = h->d_ctadt; a.Sq = Sq; a.prof = h->d_prof;
   a.num_zones = h->Z; a.num_nodes = h->nn; a.zero = 0;
   a.ph.cfl = h->params.cfl; a.ph.q_quad = h->params.q_quad; a.ph.q_lin = h->params.q_lin;
@@ -909,18 +1004,39 @@ static int host_plan(blast_cf *h) {
   return BLAST_CF_OK;
 }
 
-int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
-                       double *out_Fdot1, double *out_FTv, double *out_dt_min) {
-  if (!h) return fail(BLAST_CF_EINVAL, "handle is NULL");
-  if (!out_dt_min || ((!x || !v || !out_Fdot1) && h->nn > 0) || ((!e || !rho0detJ0 || !out_FTv) && h->Z > 0))
-    return fail(BLAST_CF_EINVAL, "NULL array argument");
-  int rc = check_async(h);
-  if (rc) return rc;
+static int host_staging(blast_cf *h) {
   const size_t nx = (size_t)h->dim * h->nn, ne = (size_t)h->Z * h->nt, nr = (size_t)h->Z * h->nq;
   if (!h->d_in) {
     CUDA_TRY(cudaMalloc(&h->d_in, (2 * nx + ne + nr + 1) * sizeof(double)));
     CUDA_TRY(cudaMalloc(&h->d_out, (nx + ne + 1) * sizeof(double)));
   }
+  return BLAST_CF_OK;
+}
+
+int blast_cf_set_rho0detJ0_host(blast_cf *h, const double *rho0detJ0) {
+  if (!h || (!rho0detJ0 && h->Z > 0)) return fail(BLAST_CF_EINVAL, "NULL argument");
+  int rc = check_async(h);
+  if (rc || (rc = host_staging(h))) return rc;
+  const size_t nx = (size_t)h->dim * h->nn, ne = (size_t)h->Z * h->nt, nr = (size_t)h->Z * h->nq;
+  double *dr = h->d_in + 2 * nx + ne;
+  if (nr) CUDA_TRY(cudaMemcpyAsync(dr, rho0detJ0, nr * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  h->rho_resident = true;
+  return BLAST_CF_OK;
+}
+
+int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                       double *out_Fdot1, double *out_FTv, double *out_dt_min) {
+  if (!h) return fail(BLAST_CF_EINVAL, "handle is NULL");
+  if (!out_dt_min || ((!x || !v || !out_Fdot1) && h->nn > 0) || ((!e || !out_FTv) && h->Z > 0))
+    return fail(BLAST_CF_EINVAL, "NULL array argument");
+  if (!rho0detJ0 && h->Z > 0 && !h->rho_resident)
+    return fail(BLAST_CF_EINVAL, "rho0detJ0 is NULL and no resident copy was set (blast_cf_set_rho0detJ0_host)");
+  int rc = check_async(h);
+  if (rc) return rc;
+  const size_t nx = (size_t)h->dim * h->nn, ne = (size_t)h->Z * h->nt, nr = (size_t)h->Z * h->nq;
+  if ((rc = host_staging(h))) return rc;
+  if (rho0detJ0) h->rho_resident = false;   // the upload below overwrites the resident copy
   if ((rc = host_plan(h))) return rc;
   blast_cf::HostPipe &P = h->hp;
   double *dx = h->d_in, *dv = dx + nx, *de = dv + nx, *dr = de + ne;
@@ -929,7 +1045,7 @@ int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const doub
     CUDA_TRY(cudaMemcpyAsync(dx, x, nx * sizeof(double), cudaMemcpyHostToDevice, h->stream));
     CUDA_TRY(cudaMemcpyAsync(dv, v, nx * sizeof(double), cudaMemcpyHostToDevice, h->stream));
     CUDA_TRY(cudaMemcpyAsync(de, e, ne * sizeof(double), cudaMemcpyHostToDevice, h->stream));
-    CUDA_TRY(cudaMemcpyAsync(dr, rho0detJ0, nr * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+    if (rho0detJ0) CUDA_TRY(cudaMemcpyAsync(dr, rho0detJ0, nr * sizeof(double), cudaMemcpyHostToDevice, h->stream));
     if ((rc = blast_cf_eval(h, dx, dv, de, dr, dF, dT, dd))) return rc;
     CUDA_TRY(cudaMemcpyAsync(out_Fdot1, dF, nx * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
     CUDA_TRY(cudaMemcpyAsync(out_FTv, dT, ne * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
@@ -942,7 +1058,7 @@ int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const doub
   CUDA_TRY(cudaStreamWaitEvent(P.s_h2d, P.ev_start, 0));
   CUDA_TRY(cudaStreamWaitEvent(P.s_d2h, P.ev_start, 0));
   KB1Args a;
-  a.zone_nodes = h->d_zone_nodes; a.J0inv = h->d_J0inv; a.zone_gamma = h->d_gamma; a.tab = h->d_tab;
+  a.zone_nodes = h->d_zone_nodes; a.J0inv = h->d_J0inv; a.J0inv_q = h->d_J0inv_q; a.zone_gamma = h->d_gamma; a.tab = h->d_tab;
   a.x = dx; a.v = dv; a.e = de; a.rho0detJ0 = dr; a.Fz1 = h->d_Fz1; a.FTv = dT; a.cta_dt = P.d_ctadt;
   a.Sq = nullptr; a.prof = nullptr; a.num_nodes = h->nn; a.zero = 0;
   a.ph.cfl = h->params.cfl; a.ph.q_quad = h->params.q_quad; a.ph.q_lin = h->params.q_lin;
@@ -961,12 +1077,15 @@ int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const doub
       done = n1;
     }
     CUDA_TRY(cudaMemcpyAsync(de + z0 * h->nt, e + z0 * h->nt, zc * h->nt * sizeof(double), cudaMemcpyHostToDevice, P.s_h2d));
-    CUDA_TRY(cudaMemcpyAsync(dr + z0 * h->nq, rho0detJ0 + z0 * h->nq, zc * h->nq * sizeof(double),
-                             cudaMemcpyHostToDevice, P.s_h2d));
+    if (rho0detJ0)
+      CUDA_TRY(cudaMemcpyAsync(dr + z0 * h->nq, rho0detJ0 + z0 * h->nq, zc * h->nq * sizeof(double),
+                               cudaMemcpyHostToDevice, P.s_h2d));
     CUDA_TRY(cudaEventRecord(P.ev_in[c], P.s_h2d));
     CUDA_TRY(cudaStreamWaitEvent(h->stream, P.ev_in[c], 0));
     KB1Args ac = a;   // the same kernel on zones [z0, z0 + zc): zone-indexed arrays shifted
-    ac.zone_nodes = h->d_zone_nodes + z0 * h->nk; ac.J0inv = h->d_J0inv + z0 * 9; ac.zone_gamma = h->d_gamma + z0;
+    ac.zone_nodes = h->d_zone_nodes + z0 * h->nk; ac.J0inv = h->d_J0inv + z0 * h->dim * h->dim;
+    ac.zone_gamma = h->d_gamma + z0;
+    if (h->d_J0inv_q) ac.J0inv_q = h->d_J0inv_q + z0 * h->nq * h->dim * h->dim;
     ac.e = de + z0 * h->nt; ac.rho0detJ0 = dr + z0 * h->nq; ac.Fz1 = h->d_Fz1 + z0 * h->dim * h->nk;
     ac.FTv = dT + z0 * h->nt; ac.cta_dt = P.d_ctadt + P.off[c]; ac.num_zones = zc;
     if (P.grid[c] > 0) h->var.launch(ac, P.grid[c], h->stream);
@@ -1046,12 +1165,13 @@ int blast_cf_eval_loopback(blast_cf *const *hs, int n, const double *const *x, c
   // 4. global min dt
   double dtg = HUGE_VAL, d;
   for (int r = 0; r < n; ++r) {
-    CUDA_TRY(cudaMemcpy(&d, out_dt_min[r], sizeof d, cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpyAsync(&d, out_dt_min[r], sizeof d, cudaMemcpyDeviceToHost, hs[r]->stream));
+    CUDA_TRY(cudaStreamSynchronize(hs[r]->stream));
     dtg = std::min(dtg, d);
   }
   // 5. ordered combine on every rank
   for (int r = 0; r < n; ++r) {
-    CUDA_TRY(cudaMemcpy(out_dt_min[r], &dtg, sizeof dtg, cudaMemcpyHostToDevice));
+    CUDA_TRY(cudaMemcpyAsync(out_dt_min[r], &dtg, sizeof dtg, cudaMemcpyHostToDevice, hs[r]->stream));
     blastcf::exchange_combine(hs[r]->xch, out_Fdot1[r]);
     CUDA_TRY(cudaStreamSynchronize(hs[r]->stream));
   }
@@ -1062,7 +1182,7 @@ int blast_cf_autotune(blast_cf *h, const double *x, const double *v, const doubl
                       double *out_Fdot1, double *out_FTv, double *out_dt_min, int reps, double *ms_out, int capacity,
                       int *num_candidates) {
   if (!h || !num_candidates) return fail(BLAST_CF_EINVAL, "NULL argument");
-  const std::vector<KB1Variant> c = kb1_candidates(h->dim, h->k);
+  const std::vector<KB1Variant> c = kb1_usable(h->dim, h->k, h->d_J0inv_q != nullptr);
   *num_candidates = (int)c.size();
   if (reps < 1) reps = 3;
   cudaEvent_t e0, e1;
@@ -1094,7 +1214,7 @@ const char *blast_cf_variant_name(const blast_cf *h, int index) {
   if (!h) return "";
   if (index < 0) return h->var.name ? h->var.name : "";
   static thread_local std::vector<KB1Variant> c;
-  c = kb1_candidates(h->dim, h->k);
+  c = kb1_usable(h->dim, h->k, h->d_J0inv_q != nullptr);
   return index < (int)c.size() ? c[index].name : "";
 }
 

@@ -819,7 +819,10 @@ int finish_setup(blast_cf_rk2 *const *S, int n) {
         return fail(BLAST_CF_EINVAL, "non-positive mass diagonal at DOF %lld of rank %d", (long long)i, r);
       d = s->fixed[i] ? 0.0 : 1.0 / d;
     }
-    if (nx > 0) CUDA_TRY(cudaMemcpy(s->invd, diag.data(), nx * sizeof(double), cudaMemcpyHostToDevice));
+    if (nx > 0) {   // ordered on the stream the CG kernels use (pageable source: wait for it)
+      CUDA_TRY(cudaMemcpyAsync(s->invd, diag.data(), nx * sizeof(double), cudaMemcpyHostToDevice, s->hv.stream));
+      CUDA_TRY(cudaStreamSynchronize(s->hv.stream));
+    }
     s->ready = true;
   }
   return BLAST_CF_OK;
@@ -1071,12 +1074,14 @@ int blast_cf_rk2_create(blast_cf *h, const blast_cf_mesh *mesh, const double *rh
     if (s->loopback) return bail(fail(BLAST_CF_EINVAL, "a loopback group needs opts->box_lo/box_hi (the global box)"));
     double mm[6] = {0, 0, 0, 0, 0, 0};
     for (int c = 0; c < D; ++c) { mm[c] = -lo[c]; mm[3 + c] = hi[c]; }
-    CUDA_TRY(cudaMemcpy(s->red, mm, 6 * sizeof(double), cudaMemcpyHostToDevice));
+    CUDA_TRY(cudaMemcpyAsync(s->red, mm, 6 * sizeof(double), cudaMemcpyHostToDevice, st));
+    CUDA_TRY(cudaStreamSynchronize(st));
     blast_cf *hh = h;
     double *rb = s->red;
     if ((rc = blastcf::group_allreduce(&hh, 1, &rb, 6, 2))) return bail(rc);
     CUDA_TRY(cudaStreamSynchronize(st));
-    CUDA_TRY(cudaMemcpy(mm, s->red, 6 * sizeof(double), cudaMemcpyDeviceToHost));
+    CUDA_TRY(cudaMemcpyAsync(mm, s->red, 6 * sizeof(double), cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(cudaStreamSynchronize(st));
     for (int c = 0; c < D; ++c) { lo[c] = -mm[c]; hi[c] = mm[3 + c]; }
   }
   s->fixed.assign(nx, 0);

@@ -18,7 +18,8 @@
 struct KB1Args {
   const double *x, *v, *e, *rho0detJ0;
   const int32_t *zone_nodes;
-  const double *J0inv;     // [Z][D*D]
+  const double *J0inv;     // [Z][D*D] per zone (affine initial zones)
+  const double *J0inv_q;   // [Z][NQ][D*D] per point (non-affine initial zones, read by the v1 kernels only), else nullptr
   const double *zone_gamma;// [Z]
   const double *tab;       // [B: N*P][G: N*P][Phi: N*T][w: N]
   double *Fz1;             // [Z][D][NK] zone-local F_z.1
@@ -223,7 +224,8 @@ __global__ void __launch_bounds__(KB1Cfg3<K, ZPC>::NTH, MINB) kb1_corner_force_3
       const double R = active ? __ldg(a.rho0detJ0 + my_z * Dm::NQ + q) : 1.0;
       const double alpha = sW[q0] * sW[q1] * sW[q2];
       PointOut<3> o;
-      point_eval3(Jm, Gv, eq, R, alpha, gamma, sJ0 + my_zl * 9, a.ph, o);
+      const double *j0p = (a.J0inv_q != nullptr && active) ? a.J0inv_q + (my_z * Dm::NQ + q) * 9 : sJ0 + my_zl * 9;
+      point_eval3(Jm, Gv, eq, R, alpha, gamma, j0p, a.ph, o);
       double *S = sRA + my_zl * Dm::SZ_A + my_qq;
 #pragma unroll
       for (int c = 0; c < 3; ++c)
@@ -453,7 +455,8 @@ __global__ void __launch_bounds__(KB1Cfg2<K, ZPC>::NTH, MINB) kb1_corner_force_2
     for (int j0 = 0; j0 < T; ++j0) eq = fma(sPhi[q0 * T + j0], Tz[2 * NF * N * P + q1 * T + j0], eq);
     const double alpha = sW[q0] * sW[q1];
     PointOut<2> o;
-    point_eval2(Jm, Gv, eq, Rq, alpha, gamma_z, sJ0 + my_zl * 4, a.ph, o);
+    const double *j0p = (a.J0inv_q != nullptr && active) ? a.J0inv_q + (my_z * NQ + my_q) * 4 : sJ0 + my_zl * 4;
+    point_eval2(Jm, Gv, eq, Rq, alpha, gamma_z, j0p, a.ph, o);
     double *S = sS + my_zl * Dm::SZ_S;
 #pragma unroll
     for (int c = 0; c < 2; ++c)

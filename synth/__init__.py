@@ -183,6 +183,22 @@ def _rho0detJ0_const(mesh: Mesh, rho_zone: np.ndarray) -> np.ndarray:
     return np.ascontiguousarray(np.repeat((rho_zone * vol)[:, None], mesh.nq, axis=1))
 
 
+RHO_POINT_AMPL = 0.25
+
+
+def _rho0detJ0_varying(mesh: Mesh, rho_zone: np.ndarray) -> np.ndarray:
+    """rho0|J0| of the S1 states: the zone value times a seeded per-point factor 1 + 0.25 (U(0,1) - 1/2).
+
+    A varying initial density inside a zone is allowed by the method (rho0|J0| is an input at every
+    quadrature point, reading R2), and it makes the parity tests see a mis-indexed point read of this
+    array.  It is a property of the initial mesh (time-invariant): its generator is seeded from the mesh
+    shape only, so the two RK2 stage states S1 / S1b of a config share it, and the x, v, e draws of S1 are
+    unchanged."""
+    rng = np.random.default_rng([7919, mesh.dim, mesh.order, *mesh.N])
+    f = 1.0 + RHO_POINT_AMPL * (rng.uniform(0.0, 1.0, size=(mesh.num_zones, mesh.nq)) - 0.5)
+    return np.ascontiguousarray(_rho0detJ0_const(mesh, rho_zone) * f)
+
+
 # ---------------------------------------------------------------------------
 # Sedov (PAPER.md:823-825; reading SURVEY §8c #16)
 # ---------------------------------------------------------------------------
@@ -214,7 +230,7 @@ def sedov_s1(mesh: Mesh, seed: int) -> State:
     rc = np.sqrt((cp ** 2).sum(0))
     e = _bump(rc) + 0.1 + 0.1 * rng.uniform(0.0, 1.0, size=rc.shape)
     return State(np.ascontiguousarray(x), np.ascontiguousarray(v), np.ascontiguousarray(e),
-                 _rho0detJ0_const(mesh, np.ones(mesh.num_zones)), name=f"S1(seed={seed})")
+                 _rho0detJ0_varying(mesh, np.ones(mesh.num_zones)), name=f"S1(seed={seed})")
 
 
 # ---------------------------------------------------------------------------
@@ -267,8 +283,9 @@ def triple_point_s1(mesh: Mesh, seed: int) -> State:
     v[0] += 0.5 * np.exp(-(((X0[0] - 1.5) / 0.3) ** 2))
     s0 = triple_point_s0(mesh)
     e = s0.e * (1.0 + 0.05 * rng.uniform(-1.0, 1.0, size=s0.e.shape))
-    return State(np.ascontiguousarray(x), np.ascontiguousarray(v), np.ascontiguousarray(e), s0.rho0detJ0,
-                 name=f"S1(seed={seed})")
+    rho, _ = _tp_rho_p(mesh)
+    return State(np.ascontiguousarray(x), np.ascontiguousarray(v), np.ascontiguousarray(e),
+                 _rho0detJ0_varying(mesh, rho), name=f"S1(seed={seed})")
 
 
 # ---------------------------------------------------------------------------
@@ -397,3 +414,43 @@ def partition(mesh: Mesh, P: int) -> List[RankPart]:
                               np.ascontiguousarray(np.concatenate(lst).astype(np.int32)) if lst else np.zeros(0, np.int32),
                               owned))
     return parts
+
+
+# ---------------------------------------------------------------------------
+# Edge-case states for the parity tests (inputs only: an affine velocity field v = B x on the current
+# nodes, shifted or scaled thermodynamic coefficients).  SURVEY §8(c) c5 names the risky regimes.
+# ---------------------------------------------------------------------------
+
+def _rotation(dim: int, rng: np.random.Generator) -> np.ndarray:
+    Q, Rr = np.linalg.qr(rng.standard_normal((dim, dim)))
+    return Q * np.sign(np.diag(Rr))
+
+
+def edge_state(mesh: Mesh, kind: str, which: str, seed: int) -> State:
+    """S1 of `kind` ("sedov" | "triple") modified into one of the regimes the parity tests must cover:
+
+    * "window":   v = B x with B = Q diag(1.5, 4, 6) 1e-12 Q^T: the smallest eigenvalue of the strain rate
+                  is 1.5e-12, inside the viscosity switch window (eps_sw, 3 eps_sw) = (1e-12, 3e-12) at every
+                  point; e scaled to ~1e-6 so the linear viscosity term is visible next to the pressure.
+    * "negative_e": S1 with every thermodynamic coefficient lowered by 0.15 (Sedov: the background
+                  e in [0.1, 0.2] straddles 0) / (triple point: by the mean coefficient): e(q) < 0 at part of the points, where the EOS clamps it to 0.
+    * "near_tie": v = B x with B = Q diag(-1, -1 + 1e-4, 0.5) Q^T: relative eigen-gap 1e-4 of the strain
+                  rate at every point, on the S1-deformed mesh (so J J0^-1 is anisotropic there).
+    """
+    base = make_state(mesh, kind, "S1", seed)
+    rng = np.random.default_rng(seed + 4242)
+    dim = mesh.dim
+    Q = _rotation(dim, rng)
+    if which == "window":
+        B = Q @ np.diag([1.5e-12, 4e-12, 6e-12][:dim]) @ Q.T
+        v = np.ascontiguousarray(B @ base.x)
+        e = np.ascontiguousarray(1e-6 * (0.5 + base.e / base.e.max()))
+        return State(base.x, v, e, base.rho0detJ0, name=f"window(seed={seed})")
+    if which == "negative_e":
+        shift = 0.15 if kind == "sedov" else float(base.e.mean())
+        return State(base.x, base.v, np.ascontiguousarray(base.e - shift), base.rho0detJ0,
+                     name=f"negative_e(seed={seed})")
+    if which == "near_tie":
+        B = Q @ np.diag([-1.0, -1.0 + 1e-4, 0.5][:dim]) @ Q.T
+        return State(base.x, np.ascontiguousarray(B @ base.x), base.e, base.rho0detJ0, name=f"near_tie(seed={seed})")
+    raise ValueError(which)

@@ -264,3 +264,50 @@ def test_rigid_rotation(orc):
     cs = np.sqrt(GAM * (GAM - 1) * E)
     dt = 0.5 * m.h[0] / (3 * cs)
     assert abs(r.dt_min - dt) < 1e-12 * dt
+
+
+@pytest.mark.parametrize("dim,k", [(2, 2), (2, 3), (3, 2)])
+def test_length_scale_orientation(orc, dim, k):
+    """l = h0 |J J0^-1 s| (reading R8) with a SHEARED initial zone and a differently sheared current zone.
+
+    Initial nodes X = A0 xi (A0 non-diagonal), current x = A1 xi, so J0 = A0 h, J = A1 h and the
+    deformation gradient J J0^-1 = A1 A0^-1 =: Fd.  v = B x with B symmetric (distinct eigenvalues):
+    grad v = B exactly (isoparametric affine field), eps = B, (lambda, s) = its smallest eigenpair
+    (numpy eigh).  e = 0 => p = 0, c_s = 0, so mu = q_quad rho l^2 |lambda| alone and
+        dt = cfl h_min^2 / (2.5 q_quad l^2 |lambda|),  h_min = sigma_min(J) / k   (numpy svd),
+        (F^T v)_j = mu (B : B) det J / k^d,  F_z.1 = Nanson with sigma = mu B.
+    The transposed / reversed products (J0^-1 J, (J J0^-1)^T, J^T J0^-T) give |. s| values that differ by
+    more than 1e-3 here (asserted), so a wrong orientation fails."""
+    A0 = np.array([[1.1, 0.35, -0.2], [0.15, 0.9, 0.25], [-0.1, 0.3, 1.2]])[:dim, :dim]
+    A1 = np.array([[1.4, -0.45, 0.3], [0.5, 0.8, -0.15], [0.2, 0.1, 0.7]])[:dim, :dim]
+    th = 0.7
+    Q = np.eye(dim)
+    Q[:2, :2] = [[np.cos(th), -np.sin(th)], [np.sin(th), np.cos(th)]]
+    if dim == 3:
+        R2 = np.array([[1, 0, 0], [0, np.cos(0.4), -np.sin(0.4)], [0, np.sin(0.4), np.cos(0.4)]])
+        Q = R2 @ Q
+    B = Q @ np.diag([-0.9, 0.2, 0.6][:dim]) @ Q.T
+    m = synth.box_mesh(dim, k, (1,) * dim)
+    box = m.x0.copy()
+    m.x0 = np.ascontiguousarray(A0 @ box)
+    x = np.ascontiguousarray(A1 @ box + 0.2)
+    v = np.ascontiguousarray(B @ x)
+    e = np.zeros((1, m.nt))
+    R = np.full((1, m.nq), np.linalg.det(A0))       # rho0 = 1
+    h0 = 0.13
+    r = orc.evaluate(m, synth.State(x, v, e, R), params=orc.Params(h0=h0))
+    lam, V = np.linalg.eigh(B)
+    s = V[:, 0]
+    Fd = A1 @ np.linalg.inv(A0)
+    ell = h0 * np.linalg.norm(Fd @ s)
+    for wrong in (np.linalg.inv(A0) @ A1, Fd.T, A1.T @ np.linalg.inv(A0).T):
+        assert abs(h0 * np.linalg.norm(wrong @ s) - ell) > 1e-3 * ell
+    rho = np.linalg.det(A0) / np.linalg.det(A1)
+    mu = 2.0 * rho * ell ** 2 * abs(lam[0])
+    hmin = np.linalg.svd(A1, compute_uv=False).min() / k
+    dt = 0.5 * hmin ** 2 / (2.5 * 2.0 * ell ** 2 * abs(lam[0]))
+    assert abs(r.dt_min - dt) < 1e-13 * dt, (r.dt_min, dt)
+    ftv = mu * (B * B).sum() * np.linalg.det(A1) / k ** dim
+    assert np.abs(r.FTv - ftv).max() < 1e-13 * abs(ftv)
+    expect = zone_F1_uniform_stress(dim, k, A1, mu * B)[:, :]
+    assert np.abs(r.Fz1[0] - expect).max() < 1e-13 * np.abs(expect).max()

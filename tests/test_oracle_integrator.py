@@ -143,3 +143,35 @@ def test_sedov_mirror_symmetry(orc):
     zp = np.arange(25).reshape(5, 5).T.reshape(-1)
     tp = np.arange(m.nt).reshape(m.order, m.order).T.reshape(-1)
     assert np.abs(e - e[zp][:, tp]).max() < 1e-12 * np.abs(e).max()
+
+
+def test_advance_step_control_sequence(orc):
+    """RK2Avg.advance's step control (reading R24), pinned on a scripted dt-estimate sequence worked out by
+    hand: reject (retry with 0.85 dt) when the estimate is below the dt used, grow by 2 % when it is at
+    least 1.25 dt, clip the last step to t_final.  step() is replaced by a stub that records the dt it was
+    given and returns the next scripted estimate, so only the control logic runs (t_final = 0.3):
+        dt 0.1      est 1.0  accept  t 0.1      next 0.102      (1.0 >= 0.125: grow)
+        dt 0.102    est 0.05 reject           next 0.0867     (0.85 dt)
+        dt 0.0867   est 0.1  accept  t 0.1867   next 0.0867     (0.1 < 0.108375: keep)
+        dt 0.0867   est 0.2  accept  t 0.2734   next 0.088434   (grow)
+        dt 0.0266   est 0.02 reject           next 0.02261    (clipped to t_final - t, then 0.85 dt)
+        dt 0.02261  est 1.0  accept  t 0.29601  next 0.0230622
+        dt 0.00399  est 1.0  accept  t 0.3      next 0.0040698  (clipped, then grown from the clipped dt)"""
+    m = synth.box_mesh(2, 1, (1, 1))
+    rk = it.RK2Avg(m, np.ones((1, m.nq)))
+    script = iter([1.0, 0.05, 0.1, 0.2, 0.02, 1.0, 1.0])
+    used = []
+
+    def stub(x, v, e, dt):
+        used.append(dt)
+        return x + dt, v, e, next(script)
+
+    rk.step = stub
+    x0 = np.zeros((2, m.num_nodes))
+    x, v, e, t, dt, steps, rejected = rk.advance(x0, x0.copy(), np.zeros((1, 1)), 0.3, 0.1, 10)
+    expect = [0.1, 0.102, 0.0867, 0.0867, 0.0266, 0.02261, 0.00399]
+    assert np.allclose(used, expect, rtol=0, atol=1e-14), used
+    assert (steps, rejected) == (5, 2)
+    assert abs(t - 0.3) < 1e-14
+    assert np.allclose(x, 0.3, atol=1e-14)   # rejected steps are not applied: x advanced by the accepted dts
+    assert abs(dt - 1.02 * 0.00399) < 1e-14
