@@ -43,9 +43,23 @@ def env_rank():
 class ClockSampler:
     """nvidia-smi clocks/throttle reasons sampled DURING the timed region (B200_PROFILING.md)."""
 
-    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+    FIELDS = ("index,clocks.sm,clocks.max.sm,{power},clocks_event_reasons.hw_slowdown,"
               "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
               "clocks_event_reasons.sw_power_cap")
+    _power_field = None
+
+    @classmethod
+    def power_field(cls):
+        """power.draw.instant where the driver has it (power.draw is a 1 s average on recent drivers)."""
+        if cls._power_field is None:
+            try:
+                r = subprocess.run(["nvidia-smi", "--query-gpu=power.draw.instant", "--format=csv,noheader"],
+                                   capture_output=True, text=True, timeout=20)
+                ok = r.returncode == 0 and "not a valid" not in (r.stdout + r.stderr).lower()
+            except Exception:
+                ok = False
+            cls._power_field = "power.draw.instant" if ok else "power.draw"
+        return cls._power_field
 
     def __init__(self, gpu_index):
         self.gpu = gpu_index
@@ -54,7 +68,8 @@ class ClockSampler:
 
     def __enter__(self):
         try:
-            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.FIELDS}",
+            fields = self.FIELDS.format(power=self.power_field())
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={fields}",
                                           "--format=csv,noheader,nounits", "-lms", "20"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
@@ -158,7 +173,7 @@ def measure_energy(gpu_index, step, stream, zones_per_step, seconds=1.5):
     n = max(10, int(seconds / max(t_step, 1e-6)))
     with ClockSampler(gpu_index) as smp:
         t_w = time.perf_counter()
-        while time.perf_counter() - t_w < 0.4:   # sampler start-up under load
+        while time.perf_counter() - t_w < 1.0:   # sampler start-up and power settling under load
             step()
             torch.cuda.synchronize()
         n_before = len(smp.lines)
@@ -179,6 +194,7 @@ def measure_energy(gpu_index, step, stream, zones_per_step, seconds=1.5):
     smi_w = statistics.mean(samples) if samples else None
     limit = meter.power_limit_w()
     out = {"window_s": secs, "steps": n, "avg_power_w": avg_w, "smi_power_w_mean": smi_w, "smi_samples": len(samples),
+           "smi_field": ClockSampler.power_field(),
            "power_limit_w": limit, "source": "NVML total-energy counter over a separate >= 1 s loop of steps"}
     if limit is not None and avg_w > limit:
         out["rejected"] = f"average {avg_w:.0f} W exceeds the {limit:.0f} W power limit"
@@ -444,7 +460,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-energy", action="store_true")
-    ap.add_argument("--energy-seconds", type=float, default=1.5)
+    ap.add_argument("--energy-seconds", type=float, default=2.0)
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

@@ -176,6 +176,19 @@ int blast_cf_get_info(const blast_cf *h, blast_cf_info *info);
 int blast_cf_set_timing(blast_cf *h, int enable);
 int blast_cf_kernel_times(blast_cf *h, float *ms3);
 
+/* Multi-rank handles: which exchange schedule eval runs.
+ * *mode = 0 (single rank), 1 (single round: KB1, KB2, then one grouped send/recv carrying the F.1 rows
+ * and each rank's dt, so no allreduce when every rank neighbours every other) or 2 (overlap: the zones
+ * touching shared nodes are numbered first — *boundary_zones of them — and their rows are exchanged on a
+ * high-priority comm stream while the interior zones compute on all but BLAST_CF_COMM_SMS (default 4)
+ * SMs; the dt allreduce(min) overlaps the node gather).  BLAST_CF_OVERLAP=0 at create forces 1.
+ * boundary_zones may be NULL. */
+int blast_cf_exchange_schedule(const blast_cf *h, int32_t *mode, int64_t *boundary_zones);
+/* Tests / profiling, overlap schedule with timing enabled: milliseconds from the start of the last eval to
+ * [0] the end of the shared-row exchange (comm stream), [1] the end of the interior zones' corner force,
+ * [2] the end of the eval.  [0] < [1] shows the exchange hidden behind the interior compute. */
+int blast_cf_debug_exchange_times(blast_cf *h, float *ms3);
+
 /* Tests only: the per-CTA minimum dt of the last eval, copied to host_out[capacity] after synchronizing
  * the stream (host_out NULL: only report the sizes).  Zone z belongs to CTA (z / zones_per_cta) mod num_ctas
  * (the corner-force kernel walks zone batches c, c + num_ctas, ... per CTA). */

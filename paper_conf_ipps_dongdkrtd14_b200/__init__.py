@@ -90,6 +90,8 @@ def lib():
     L.blast_cf_eval.argtypes = [vp] * 8
     L.blast_cf_eval_host.argtypes = [vp] * 8
     L.blast_cf_set_rho0detJ0_host.argtypes = [vp, vp]
+    L.blast_cf_exchange_schedule.argtypes = [vp, ctypes.POINTER(i32), ctypes.POINTER(i64)]
+    L.blast_cf_debug_exchange_times.argtypes = [vp, ctypes.POINTER(ctypes.c_float)]
     L.blast_cf_eval_debug_Fz.argtypes = [vp] * 6
     L.blast_cf_get_info.argtypes = [vp, ctypes.POINTER(Info)]
     L.blast_cf_set_timing.argtypes = [vp, ctypes.c_int]
@@ -123,7 +125,8 @@ def lib():
     for f in ("blast_cf_rk2_create", "blast_cf_rk2_step", "blast_cf_rk2_rates", "blast_cf_rk2_mass_apply",
               "blast_cf_rk2_energy", "blast_cf_rk2_destroy", "blast_cf_rk2_advance", "blast_cf_rk2_setup_loopback",
               "blast_cf_rk2_rates_loopback", "blast_cf_rk2_energy_loopback",
-              "blast_cf_create", "blast_cf_eval", "blast_cf_eval_host", "blast_cf_set_rho0detJ0_host", "blast_cf_eval_debug_Fz", "blast_cf_get_info",
+              "blast_cf_create", "blast_cf_eval", "blast_cf_eval_host", "blast_cf_set_rho0detJ0_host",
+              "blast_cf_exchange_schedule", "blast_cf_debug_exchange_times", "blast_cf_eval_debug_Fz", "blast_cf_get_info",
               "blast_cf_set_timing", "blast_cf_kernel_times", "blast_cf_destroy", "blast_cf_nccl_unique_id_size",
               "blast_cf_nccl_get_unique_id", "blast_cf_exchange_plan", "blast_cf_owner_mask", "blast_cf_debug_cta_dt",
               "blast_cf_debug_stage_clocks", "blast_cf_eval_loopback", "blast_cf_autotune"):
@@ -351,6 +354,17 @@ class CornerForce:
         out = np.zeros((n, 16), dtype=np.int64)
         _check(lib().blast_cf_debug_stage_clocks(self._h, out.ctypes.data, out.size), "blast_cf_debug_stage_clocks")
         return out
+
+    def exchange_schedule(self):
+        """(0 single rank | 1 single round | 2 overlap, number of boundary zones) — blast_cf_exchange_schedule."""
+        nb, mode = ctypes.c_int64(0), ctypes.c_int32(0)
+        _check(lib().blast_cf_exchange_schedule(self._h, ctypes.byref(mode), ctypes.byref(nb)), "blast_cf_exchange_schedule")
+        return mode.value, nb.value
+
+    def debug_exchange_times(self):
+        ms = (ctypes.c_float * 3)()
+        _check(lib().blast_cf_debug_exchange_times(self._h, ms), "blast_cf_debug_exchange_times")
+        return list(ms)
 
     def set_timing(self, enable: bool):
         _check(lib().blast_cf_set_timing(self._h, int(enable)), "blast_cf_set_timing")

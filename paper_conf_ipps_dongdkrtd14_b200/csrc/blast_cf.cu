@@ -414,9 +414,43 @@ int exchange_create(Exchange **out, const blast_cf_mesh *mesh, int dim, int64_t 
   }
   if (cudaMalloc(&x->d_send, std::max<int64_t>(total * dim, 1) * sizeof(double)) != cudaSuccess ||
       cudaMalloc(&x->d_recv, std::max<int64_t>(total * dim, 1) * sizeof(double)) != cudaSuccess ||
-      cudaMalloc(&x->d_tmp, 2 * sizeof(double)) != cudaSuccess) {
+      cudaMalloc(&x->d_tmp, 2 * sizeof(double)) != cudaSuccess ||
+      cudaMalloc(&x->d_rdt, std::max(x->num_nbr, 1) * sizeof(double)) != cudaSuccess) {
     exchange_destroy(x);
     return fail(BLAST_CF_ENOMEM, "exchange buffers");
+  }
+  // overlap schedule: possible when the zones touching shared nodes are exactly the prefix [0, nb)
+  {
+    int nk = 1;
+    for (int d = 0; d < dim; ++d) nk *= mesh->order + 1;
+    std::vector<char> shared((size_t)std::max<int64_t>(nn, 1), 0);
+    for (int64_t r = 0; r < total; ++r) shared[mesh->nbr_nodes[r]] = 1;
+    int64_t nb = 0;
+    bool prefix = true;
+    for (int64_t z = 0; z < mesh->num_zones; ++z) {
+      bool b = false;
+      for (int a = 0; a < nk && !b; ++a) b = shared[mesh->zone_nodes[z * nk + a]] != 0;
+      if (b) {
+        if (nb != z) prefix = false;
+        ++nb;
+      }
+    }
+    const char *ov = getenv("BLAST_CF_OVERLAP");
+    x->nb = nb;
+    x->overlap = prefix && nb > 0 && nb < mesh->num_zones && !(ov && ov[0] == '0');
+  }
+  {
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);   // hi = greatest priority (numerically lowest)
+    if (cudaStreamCreateWithPriority(&x->s_comm, cudaStreamNonBlocking, hi) != cudaSuccess ||
+        cudaEventCreateWithFlags(&x->ev_b, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&x->ev_i, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&x->ev_p, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&x->ev_x, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreate(&x->ev_sent) != cudaSuccess) {
+      exchange_destroy(x);
+      return fail(BLAST_CF_ECUDA, "exchange stream / events");
+    }
   }
   if (!uid) {
     *out = x;
@@ -460,19 +494,38 @@ void exchange_combine(Exchange *x, double *F1) {
   }
 }
 
-int exchange_run(Exchange *x, double *F1, double *dt) {
+// grouped ncclSend / ncclRecv of every neighbour's shared rows on stream st; with_dt: each rank's dt (one
+// double) travels in the same group (the single-round schedule's piggy-backed min dt)
+int exchange_send_rows(Exchange *x, cudaStream_t st, bool with_dt, const double *dt) {
   const int dim = x->dim;
-  if (!x->comm) return BLAST_CF_OK;   // loopback: blast_cf_eval_loopback moves the data
-  exchange_pack(x, F1);
   NCCL_TRY(x->api->GroupStart(), "ncclGroupStart");
   for (int i = 0; i < x->num_nbr; ++i) {
     const int64_t o = x->nbr_offset[i], cnt = x->nbr_offset[i + 1] - o;
-    if (cnt == 0) continue;
-    NCCL_TRY(x->api->Send(x->d_send + o * dim, (size_t)cnt * dim, ncclDouble, x->nbr_rank[i], x->comm, x->stream), "ncclSend");
-    NCCL_TRY(x->api->Recv(x->d_recv + o * dim, (size_t)cnt * dim, ncclDouble, x->nbr_rank[i], x->comm, x->stream), "ncclRecv");
+    if (cnt > 0) {
+      NCCL_TRY(x->api->Send(x->d_send + o * dim, (size_t)cnt * dim, ncclDouble, x->nbr_rank[i], x->comm, st), "ncclSend");
+      NCCL_TRY(x->api->Recv(x->d_recv + o * dim, (size_t)cnt * dim, ncclDouble, x->nbr_rank[i], x->comm, st), "ncclRecv");
+    }
+    if (with_dt) {
+      NCCL_TRY(x->api->Send(dt, 1, ncclDouble, x->nbr_rank[i], x->comm, st), "ncclSend(dt)");
+      NCCL_TRY(x->api->Recv(x->d_rdt + i, 1, ncclDouble, x->nbr_rank[i], x->comm, st), "ncclRecv(dt)");
+    }
   }
   NCCL_TRY(x->api->GroupEnd(), "ncclGroupEnd");
-  NCCL_TRY(x->api->AllReduce(dt, dt, 1, ncclDouble, ncclMin, x->comm, x->stream), "ncclAllReduce(min dt)");
+  return BLAST_CF_OK;
+}
+
+// single-round schedule, after KB2 (F1 = this rank's partial F.1, dt = its local min dt)
+int exchange_run(Exchange *x, double *F1, double *dt) {
+  if (!x->comm) return BLAST_CF_OK;   // loopback: blast_cf_eval_loopback moves the data
+  exchange_pack(x, F1);
+  const bool all_nbrs = x->num_nbr == x->nranks - 1;   // then the neighbours' dts are every rank's dt
+  int rc = exchange_send_rows(x, x->stream, all_nbrs, dt);
+  if (rc) return rc;
+  if (all_nbrs) {
+    if (x->num_nbr > 0) xch_dt_combine<<<1, 32, 0, x->stream>>>(dt, x->d_rdt, x->num_nbr);
+  } else {
+    NCCL_TRY(x->api->AllReduce(dt, dt, 1, ncclDouble, ncclMin, x->comm, x->stream), "ncclAllReduce(min dt)");
+  }
   exchange_combine(x, F1);
   return BLAST_CF_OK;
 }
@@ -487,7 +540,7 @@ struct blast_cf {
   cudaStream_t stream = nullptr;
   int device = 0;
   KB1Variant var{};
-  int ncta = 0, regs = 0, local_bytes = 0;
+  int ncta = 0, regs = 0, local_bytes = 0, sms = 148;
   int64_t ncta_cap = 0;
   // device memory
   double *d_tab = nullptr, *d_J0inv = nullptr, *d_gamma = nullptr, *d_Fz1 = nullptr, *d_ctadt = nullptr;
@@ -547,6 +600,7 @@ int apply_variant(blast_cf *h, const KB1Variant &v) {
     h->local_bytes = (int)fa.localSizeBytes;
   }
   h->var = v;
+  cudaDeviceGetAttribute(&h->sms, cudaDevAttrMultiProcessorCount, h->device);
   h->ncta = (int)((h->Z + v.zpc - 1) / v.zpc);
   if (v.persistent && h->ncta > 0) {
     int occ = 0, sms = 0;
@@ -781,7 +835,7 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
       (rc = upload(&h->d_ptr, ptr.data(), ptr.size())) || (rc = upload(&h->d_ent, ent.data(), ent.size())))
     return bail(rc);
   if (cudaMalloc(&h->d_Fz1, std::max<size_t>((size_t)Z * dim * nk, 1) * sizeof(double)) != cudaSuccess ||
-      cudaMalloc(&h->d_ctadt, std::max<int64_t>(h->ncta_cap, 1) * sizeof(double)) != cudaSuccess)
+      cudaMalloc(&h->d_ctadt, (std::max<int64_t>(h->ncta_cap, 1) + 2) * sizeof(double)) != cudaSuccess)
     return bail(fail(BLAST_CF_ENOMEM, "workspace allocation"));
   for (auto &e : h->ev)
     if (cudaEventCreate(&e) != cudaSuccess) return bail(fail(BLAST_CF_ECUDA, "event create"));
@@ -791,13 +845,8 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
   return BLAST_CF_OK;
 }
 
-static int eval_impl(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
-                     double *out_Fdot1, double *out_FTv, double *out_dt_min, double *Sq) {
-  if (!h) return fail(BLAST_CF_EINVAL, "handle is NULL");
-  if (!out_dt_min || ((!x || !v || !out_Fdot1) && h->nn > 0) || ((!e || !rho0detJ0 || !out_FTv) && h->Z > 0))
-    return fail(BLAST_CF_EINVAL, "NULL array argument");
-  int rc = check_async(h);
-  if (rc) return rc;
+static KB1Args make_args(const blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                         double *out_FTv, double *Sq) {
   KB1Args a;
   a.x = x; a.v = v; a.e = e; a.rho0detJ0 = rho0detJ0;
   a.zone_nodes = h->d_zone_nodes; a.J0inv = h->d_J0inv; a.J0inv_q = h->d_J0inv_q; a.zone_gamma = h->d_gamma; a.tab = h->d_tab;
@@ -806,19 +855,101 @@ static int eval_impl(blast_cf *h, const double *x, const double *v, const double
   a.ph.cfl = h->params.cfl; a.ph.q_quad = h->params.q_quad; a.ph.q_lin = h->params.q_lin;
   a.ph.eps_sw = h->params.eps_switch; a.ph.inv_2eps = 0.5 / h->params.eps_switch; a.ph.h0 = h->h0; a.ph.k = (double)h->k;
   a.ph.use_visc = h->params.use_viscosity; a.ph.use_vort = h->params.use_vorticity;
-  if (h->timing) cudaEventRecord(h->ev[0], h->stream);
-  if (h->ncta > 0) h->var.launch(a, h->ncta, h->stream);
-  if (h->timing) cudaEventRecord(h->ev[1], h->stream);
+  return a;
+}
+
+// KB1 on the zone range [z0, z0 + zc) (zone-indexed pointers shifted), per-CTA dt slots from slot_off
+static void launch_range(const blast_cf *h, const KB1Args &base, int64_t z0, int64_t zc, int grid, int slot_off,
+                         cudaStream_t st) {
+  if (zc <= 0 || grid <= 0) return;
+  KB1Args ac = base;
+  const int dd = h->dim * h->dim;
+  ac.zone_nodes = h->d_zone_nodes + z0 * h->nk; ac.J0inv = h->d_J0inv + z0 * dd; ac.zone_gamma = h->d_gamma + z0;
+  if (base.J0inv_q) ac.J0inv_q = base.J0inv_q + z0 * h->nq * dd;
+  if (base.Sq) ac.Sq = base.Sq + z0 * h->nq * dd;
+  ac.e = base.e + z0 * h->nt; ac.rho0detJ0 = base.rho0detJ0 + z0 * h->nq; ac.Fz1 = h->d_Fz1 + z0 * h->dim * h->nk;
+  ac.FTv = base.FTv + z0 * h->nt; ac.cta_dt = h->d_ctadt + slot_off; ac.num_zones = zc; ac.prof = nullptr;
+  h->var.launch(ac, grid, st);
+}
+
+// grid of a range launch; `reserve`: persistent kernels leave that many SMs' worth of CTAs to the comm stream
+static int range_grid(const blast_cf *h, int64_t zc, int reserve_sms) {
+  int64_t g = (zc + h->var.zpc - 1) / h->var.zpc;
+  if (h->var.persistent) {
+    int cap = h->ncta;
+    if (reserve_sms > 0 && h->sms > reserve_sms) cap -= (int)(((int64_t)reserve_sms * h->ncta + h->sms - 1) / h->sms);
+    g = std::min<int64_t>(g, std::max(cap, 1));
+  }
+  return (int)g;
+}
+
+static int comm_sms() {
+  const char *e = getenv("BLAST_CF_COMM_SMS");
+  return e ? std::max(0, atoi(e)) : 4;
+}
+
+static void launch_kb2(const blast_cf *h, double *F1, const double *cta_dt, int ncta, double *dt, cudaStream_t st) {
   const int gthreads = 256;
   const int64_t gblocks = std::max<int64_t>(1, (h->nn + gthreads - 1) / gthreads);
   if (h->dim == 3)
-    kb2_gather<3, 8><<<(unsigned)gblocks, gthreads, 0, h->stream>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->nk,
-                                                                     out_Fdot1, h->d_ctadt, h->ncta, out_dt_min);
+    kb2_gather<3, 8><<<(unsigned)gblocks, gthreads, 0, st>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->nk, F1, cta_dt, ncta, dt);
   else
-    kb2_gather<2, 4><<<(unsigned)gblocks, gthreads, 0, h->stream>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->nk,
-                                                                     out_Fdot1, h->d_ctadt, h->ncta, out_dt_min);
+    kb2_gather<2, 4><<<(unsigned)gblocks, gthreads, 0, st>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->nk, F1, cta_dt, ncta, dt);
+}
+
+static void launch_pack_gather(const blast_cf *h, cudaStream_t st) {
+  const blastcf::Exchange *x = h->xch;
+  if (x->nrows <= 0) return;
+  const int blocks = (int)std::min<int64_t>((x->nrows + 127) / 128, 1184);
+  blastcf::xch_pack_gather<<<blocks, 128, 0, st>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nk, h->dim, x->d_rows, x->nrows,
+                                                   x->d_send);
+}
+
+// Overlap schedule of a multi-rank NCCL handle: boundary zones, then the exchange of their
+// shared rows on the comm stream while the interior zones compute; the dt allreduce overlaps KB2.
+static int eval_overlap(blast_cf *h, const KB1Args &a, double *out_Fdot1, double *out_dt_min) {
+  blastcf::Exchange *x = h->xch;
+  const int64_t nb = x->nb, ni = h->Z - nb;
+  const int gb = range_grid(h, nb, 0), gi = range_grid(h, ni, comm_sms());
+  if (h->timing) cudaEventRecord(h->ev[0], h->stream);
+  launch_range(h, a, 0, nb, gb, 0, h->stream);
+  CUDA_TRY(cudaEventRecord(x->ev_b, h->stream));
+  CUDA_TRY(cudaStreamWaitEvent(x->s_comm, x->ev_b, 0));
+  launch_pack_gather(h, x->s_comm);
+  int rc = blastcf::exchange_send_rows(x, x->s_comm, false, nullptr);
+  if (rc) return rc;
+  if (h->timing) cudaEventRecord(x->ev_sent, x->s_comm);
+  launch_range(h, a, nb, ni, gi, gb, h->stream);
+  CUDA_TRY(cudaEventRecord(x->ev_i, h->stream));
+  if (h->timing) cudaEventRecord(h->ev[1], h->stream);
+  CUDA_TRY(cudaStreamWaitEvent(x->s_comm, x->ev_i, 0));
+  blastcf::xch_dt_reduce<<<1, 256, 0, x->s_comm>>>(h->d_ctadt, gb + gi, out_dt_min);
+  if (x->api->AllReduce(out_dt_min, out_dt_min, 1, ncclDouble, ncclMin, x->comm, x->s_comm) != ncclSuccess)
+    return fail(BLAST_CF_ENCCL, "ncclAllReduce(min dt)");
+  CUDA_TRY(cudaEventRecord(x->ev_x, x->s_comm));
+  launch_kb2(h, out_Fdot1, nullptr, 0, x->d_tmp, h->stream);   // node gather; dt comes from the comm stream
   if (h->timing) cudaEventRecord(h->ev[2], h->stream);
-  if (h->xch) {
+  CUDA_TRY(cudaStreamWaitEvent(h->stream, x->ev_x, 0));
+  blastcf::exchange_combine(x, out_Fdot1);
+  if (h->timing) cudaEventRecord(h->ev[3], h->stream);
+  return check_async(h);
+}
+
+static int eval_impl(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
+                     double *out_Fdot1, double *out_FTv, double *out_dt_min, double *Sq) {
+  if (!h) return fail(BLAST_CF_EINVAL, "handle is NULL");
+  if (!out_dt_min || ((!x || !v || !out_Fdot1) && h->nn > 0) || ((!e || !rho0detJ0 || !out_FTv) && h->Z > 0))
+    return fail(BLAST_CF_EINVAL, "NULL array argument");
+  int rc = check_async(h);
+  if (rc) return rc;
+  const KB1Args a = make_args(h, x, v, e, rho0detJ0, out_FTv, Sq);
+  if (h->xch && h->xch->comm && h->xch->overlap) return eval_overlap(h, a, out_Fdot1, out_dt_min);
+  if (h->timing) cudaEventRecord(h->ev[0], h->stream);
+  if (h->ncta > 0) h->var.launch(a, h->ncta, h->stream);
+  if (h->timing) cudaEventRecord(h->ev[1], h->stream);
+  launch_kb2(h, out_Fdot1, h->d_ctadt, h->ncta, out_dt_min, h->stream);
+  if (h->timing) cudaEventRecord(h->ev[2], h->stream);
+  if (h->xch) {   // single-round schedule (a loopback handle: local part only, blast_cf_eval_loopback exchanges)
     rc = blastcf::exchange_run(h->xch, out_Fdot1, out_dt_min);
     if (rc) return rc;
   }
@@ -1139,6 +1270,73 @@ int blast_cf_eval_loopback(blast_cf *const *hs, int n, const double *const *x, c
       return fail(BLAST_CF_EINVAL, "handle %d is not rank %d of a %d-rank loopback group", r, r, n);
   }
   int rc;
+  bool all_overlap = true;
+  for (int r = 0; r < n; ++r) all_overlap = all_overlap && hs[r]->xch->overlap;
+  if (all_overlap) {
+    // the overlap schedule of the NCCL path with device copies for the messages: per rank, KB1 on its
+    // boundary zones, then (comm stream) the pack of its shared rows; the copies of a rank's recv rows wait
+    // for its neighbours' packs; KB1 on the interior zones runs meanwhile on the rank's own stream
+    std::vector<KB1Args> as(n);
+    std::vector<int> gb(n), gi(n);
+    for (int r = 0; r < n; ++r) {
+      blast_cf *h = hs[r];
+      if ((rc = check_async(h))) return rc;
+      as[r] = make_args(h, x[r], v[r], e[r], rho0detJ0[r], out_FTv[r], nullptr);
+      gb[r] = range_grid(h, h->xch->nb, 0);
+      gi[r] = range_grid(h, h->Z - h->xch->nb, comm_sms());
+      if (h->timing) cudaEventRecord(h->ev[0], h->stream);
+      launch_range(h, as[r], 0, h->xch->nb, gb[r], 0, h->stream);
+      CUDA_TRY(cudaEventRecord(h->xch->ev_b, h->stream));
+      CUDA_TRY(cudaStreamWaitEvent(h->xch->s_comm, h->xch->ev_b, 0));
+      launch_pack_gather(h, h->xch->s_comm);
+      CUDA_TRY(cudaEventRecord(h->xch->ev_p, h->xch->s_comm));
+    }
+    for (int r = 0; r < n; ++r) {   // "send / recv": rank r's recv rows from q are q's send rows for r
+      blastcf::Exchange *xr = hs[r]->xch;
+      for (int i = 0; i < xr->num_nbr; ++i) {
+        const int q = xr->nbr_rank[i];
+        blastcf::Exchange *xq = hs[q]->xch;
+        int iq = -1;
+        for (int t = 0; t < xq->num_nbr; ++t)
+          if (xq->nbr_rank[t] == r) iq = t;
+        const int64_t cnt = xr->nbr_offset[i + 1] - xr->nbr_offset[i];
+        if (iq < 0 || xq->nbr_offset[iq + 1] - xq->nbr_offset[iq] != cnt)
+          return fail(BLAST_CF_EINVAL, "ranks %d and %d disagree on their shared nodes", r, q);
+        CUDA_TRY(cudaStreamWaitEvent(xr->s_comm, xq->ev_p, 0));
+        CUDA_TRY(cudaMemcpyAsync(xr->d_recv + xr->nbr_offset[i] * xr->dim, xq->d_send + xq->nbr_offset[iq] * xq->dim,
+                                 cnt * xr->dim * sizeof(double), cudaMemcpyDeviceToDevice, xr->s_comm));
+      }
+      if (hs[r]->timing) cudaEventRecord(xr->ev_sent, xr->s_comm);
+    }
+    for (int r = 0; r < n; ++r) {
+      blast_cf *h = hs[r];
+      blastcf::Exchange *xr = h->xch;
+      launch_range(h, as[r], xr->nb, h->Z - xr->nb, gi[r], gb[r], h->stream);
+      CUDA_TRY(cudaEventRecord(xr->ev_i, h->stream));
+      if (h->timing) cudaEventRecord(h->ev[1], h->stream);
+      CUDA_TRY(cudaStreamWaitEvent(xr->s_comm, xr->ev_i, 0));
+      blastcf::xch_dt_reduce<<<1, 256, 0, xr->s_comm>>>(h->d_ctadt, gb[r] + gi[r], out_dt_min[r]);
+      CUDA_TRY(cudaEventRecord(xr->ev_x, xr->s_comm));
+      launch_kb2(h, out_Fdot1[r], nullptr, 0, xr->d_tmp, h->stream);
+      if (h->timing) cudaEventRecord(h->ev[2], h->stream);
+    }
+    double dtg = HUGE_VAL, d;   // the allreduce(min): on the host in a loopback group
+    for (int r = 0; r < n; ++r) {
+      CUDA_TRY(cudaStreamSynchronize(hs[r]->xch->s_comm));
+      CUDA_TRY(cudaMemcpyAsync(&d, out_dt_min[r], sizeof d, cudaMemcpyDeviceToHost, hs[r]->xch->s_comm));
+      CUDA_TRY(cudaStreamSynchronize(hs[r]->xch->s_comm));
+      dtg = std::min(dtg, d);
+    }
+    for (int r = 0; r < n; ++r) {
+      blast_cf *h = hs[r];
+      CUDA_TRY(cudaMemcpyAsync(out_dt_min[r], &dtg, sizeof dtg, cudaMemcpyHostToDevice, h->stream));
+      CUDA_TRY(cudaStreamWaitEvent(h->stream, h->xch->ev_x, 0));
+      blastcf::exchange_combine(h->xch, out_Fdot1[r]);
+      if (h->timing) cudaEventRecord(h->ev[3], h->stream);
+      CUDA_TRY(cudaStreamSynchronize(h->stream));
+    }
+    return check_async(hs[0]);
+  }
   // 1. local corner force + gather on every partition, 2. pack shared-node partials
   for (int r = 0; r < n; ++r) {
     if ((rc = eval_impl(hs[r], x[r], v[r], e[r], rho0detJ0[r], out_Fdot1[r], out_FTv[r], out_dt_min[r], nullptr)))
@@ -1234,6 +1432,23 @@ int blast_cf_get_info(const blast_cf *h, blast_cf_info *info) {
 int blast_cf_set_timing(blast_cf *h, int enable) {
   if (!h) return fail(BLAST_CF_EINVAL, "handle is NULL");
   h->timing = enable != 0;
+  return BLAST_CF_OK;
+}
+
+int blast_cf_debug_exchange_times(blast_cf *h, float *ms3) {
+  if (!h || !ms3) return fail(BLAST_CF_EINVAL, "NULL argument");
+  if (!h->timing || !h->xch || !h->xch->overlap) return fail(BLAST_CF_EINVAL, "timing off or no overlap schedule");
+  CUDA_TRY(cudaEventSynchronize(h->ev[3]));
+  CUDA_TRY(cudaEventElapsedTime(&ms3[0], h->ev[0], h->xch->ev_sent));
+  CUDA_TRY(cudaEventElapsedTime(&ms3[1], h->ev[0], h->ev[1]));
+  CUDA_TRY(cudaEventElapsedTime(&ms3[2], h->ev[0], h->ev[3]));
+  return BLAST_CF_OK;
+}
+
+int blast_cf_exchange_schedule(const blast_cf *h, int32_t *mode, int64_t *boundary_zones) {
+  if (!h || !mode) return fail(BLAST_CF_EINVAL, "NULL argument");
+  *mode = h->xch ? (h->xch->overlap ? 2 : 1) : 0;
+  if (boundary_zones) *boundary_zones = h->xch ? h->xch->nb : 0;
   return BLAST_CF_OK;
 }
 

@@ -7,7 +7,14 @@
 //   2. exchanges them with grouped ncclSend / ncclRecv on the handle's stream,
 //   3. sums, for every shared node, the partials of all sharing ranks in ASCENDING RANK order, so every
 //      sharer ends with bitwise identical values (reading R20),
-// and takes the global min dt with ncclAllReduce(min).
+// and takes the global min dt.  Two schedules:
+//   overlap (zones numbered boundary-first): KB1 on the boundary zones; on a high-priority comm stream the
+//     shared rows are gathered from the zone-local buffer and exchanged while KB1 runs on the interior
+//     zones (on all but a few SMs, left to the pack and NCCL kernels); the dt allreduce(min) then overlaps
+//     KB2; the ordered combine closes the eval;
+//   single round (any numbering): KB1, KB2, then ONE grouped send/recv that carries each rank's dt next to
+//     its F.1 rows (every rank of the block partitions neighbours every other, so no allreduce is needed;
+//     otherwise an allreduce(min) follows).
 // NCCL is loaded with dlopen at create time so that single-GPU use never touches it.
 #pragma once
 #include <dlfcn.h>
@@ -138,6 +145,49 @@ __global__ void xch_combine(double *__restrict__ F1, int64_t nn, int dim, const 
   }
 }
 
+// Overlap schedule (boundary zones first): the partial F.1 of a shared row straight from the zone-local
+// buffer, summed over the node's CSR entries in ascending zone id — the same order, hence the same bits,
+// as KB2's gather of that node (every zone touching a shared node is a boundary zone).
+__global__ void xch_pack_gather(const double *__restrict__ Fz1, const int32_t *__restrict__ ptr,
+                                const int32_t *__restrict__ ent, int nk, int dim, const int32_t *__restrict__ rows,
+                                int64_t nrows, double *__restrict__ send) {
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < nrows; r += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t node = rows[r];
+    double s[3] = {0.0, 0.0, 0.0};
+    for (int i = ptr[node]; i < ptr[node + 1]; ++i) {
+      const int o = ent[i];
+      for (int c = 0; c < dim; ++c) s[c] += Fz1[o + c * nk];
+    }
+    for (int c = 0; c < dim; ++c) send[r * dim + c] = s[c];
+  }
+}
+
+// min over the per-CTA dt slots of this rank's corner-force launches (one block)
+__global__ void xch_dt_reduce(const double *__restrict__ cta_dt, int n, double *__restrict__ out) {
+  __shared__ double red[32];
+  double m = __longlong_as_double(0x7ff0000000000000LL);
+  for (int i = threadIdx.x; i < n; i += blockDim.x) m = fmin(m, cta_dt[i]);
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) m = fmin(m, __shfl_xor_sync(0xffffffffu, m, o));
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = m;
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    double r = threadIdx.x < (blockDim.x >> 5) ? red[threadIdx.x] : __longlong_as_double(0x7ff0000000000000LL);
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) r = fmin(r, __shfl_xor_sync(0xffffffffu, r, o));
+    if (threadIdx.x == 0) *out = r;
+  }
+}
+
+// single-round schedule: dt = min(own, every neighbour's dt received with its F.1 rows)
+__global__ void xch_dt_combine(double *__restrict__ dt, const double *__restrict__ recv_dt, int n) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    double m = *dt;
+    for (int i = 0; i < n; ++i) m = fmin(m, recv_dt[i]);
+    *dt = m;
+  }
+}
+
 struct Exchange {
   NcclApi *api = nullptr;
   ncclComm_t comm = nullptr;
@@ -150,22 +200,36 @@ struct Exchange {
   int32_t *d_rows = nullptr, *d_unodes = nullptr;
   int64_t *d_sptr = nullptr, *d_src = nullptr;
   double *d_send = nullptr, *d_recv = nullptr, *d_tmp = nullptr;
+  double *d_rdt = nullptr;       // [num_nbr] neighbours' dt (single-round schedule)
+  // overlap schedule: zones [0, nb) touch shared nodes (boundary), [nb, Z) do not (interior)
+  bool overlap = false;
+  int64_t nb = 0;
+  cudaStream_t s_comm = nullptr;   // high-priority stream of the pack / NCCL / dt work
+  cudaEvent_t ev_b = nullptr, ev_i = nullptr, ev_p = nullptr, ev_x = nullptr, ev_sent = nullptr;
 };
 
 inline void exchange_destroy(Exchange *x) {
   if (!x) return;
   if (x->comm && x->api) x->api->CommDestroy(x->comm);
   cudaFree(x->d_rows); cudaFree(x->d_unodes); cudaFree(x->d_sptr); cudaFree(x->d_src);
-  cudaFree(x->d_send); cudaFree(x->d_recv); cudaFree(x->d_tmp);
+  cudaFree(x->d_send); cudaFree(x->d_recv); cudaFree(x->d_tmp); cudaFree(x->d_rdt);
+  for (cudaEvent_t e : {x->ev_b, x->ev_i, x->ev_p, x->ev_x, x->ev_sent})
+    if (e) cudaEventDestroy(e);
+  if (x->s_comm) cudaStreamDestroy(x->s_comm);
   delete x;
 }
 
-inline int exchange_kernels(const Exchange *x) { return (x->nrows > 0 ? 1 : 0) + (x->nu > 0 ? 1 : 0); }
+// kernels of ours one eval launches besides KB1 / KB2 (NCCL's own kernels not counted)
+inline int exchange_kernels(const Exchange *x) {
+  const int combine = x->nu > 0 ? 1 : 0, pack = x->nrows > 0 ? 1 : 0;
+  return x->overlap ? 1 /* second KB1 launch */ + pack + 1 /* dt reduce */ + combine : pack + combine + 1 /* dt combine */;
+}
 
 int exchange_create(Exchange **out, const blast_cf_mesh *mesh, int dim, int64_t nn, cudaStream_t stream,
                     const void *uid);
 int exchange_allreduce_sum2(Exchange *x, double *a, double *b);
 int exchange_run(Exchange *x, double *F1, double *dt);
+int exchange_send_rows(Exchange *x, cudaStream_t st, bool with_dt, const double *dt);
 void exchange_pack(Exchange *x, const double *F1);
 void exchange_combine(Exchange *x, double *F1);
 int nccl_get_unique_id(void *out);

@@ -86,8 +86,12 @@ def _check_de(o, r, vbar, de, de0):
     Vz = vbar[:, o.mesh.zone_nodes].transpose(1, 0, 2).reshape(Z, -1)
     FTV = np.einsum("zij,zi->zj", r.Fz, Vz)
     res = np.einsum("zij,zj->zi", o.masses.ME, de) - FTV
-    assert np.abs(res).max() < 1e-12 * np.abs(FTV).max()
     cond = max(np.linalg.cond(o.masses.ME[z]) for z in range(min(Z, 4)))
+    # An explicit inverse is not backward stable: fl(M^-1) b has residual up to ~cond(M) eps |b|, so the
+    # residual bar is 1e-12 only while cond(M_E) eps stays below it (zone-constant rho0|J0|: the tensor
+    # path; the per-point rho0|J0| of the S1 states takes the dense per-zone inverse, cond up to 4e7 at
+    # 2D k = 8).
+    assert np.abs(res).max() < max(1e-12, 20 * cond * 2.2e-16) * np.abs(FTV).max(), cond
     assert rel(de, de0) < max(1e-12, 20 * cond * 2.2e-16), (rel(de, de0), cond)
 
 

@@ -9,13 +9,17 @@ import synth
 pytestmark = pytest.mark.gpu
 
 
+@pytest.mark.parametrize("overlap", ["1", "0"])
 @pytest.mark.parametrize("name,N,k,P", [("C3", (4, 4, 4), None, 2), ("C3", (4, 4, 4), None, 8),
                                         ("C4", (4, 3, 2), None, 4), ("C2", (8, 6), 3, 8), ("C1", None, None, 4),
-                                        ("C5", (4, 2, 2), None, 8)])
-def test_loopback_exchange(orc, name, N, k, P):
+                                        ("C5", (4, 2, 2), None, 8), ("C3", (8, 6, 6), None, 8), ("C2", (12, 10), 4, 4)])
+def test_loopback_exchange(orc, name, N, k, P, overlap, monkeypatch):
+    """Both exchange schedules (overlap: boundary zones, exchange on the comm stream while the interior
+    zones compute; single round) give the single-domain result on every node."""
     import torch
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
+    monkeypatch.setenv("BLAST_CF_OVERLAP", overlap)
     import paper_conf_ipps_dongdkrtd14_b200 as cf
     m, s = synth.config(name, "S1", N=N, k=k)
     t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
@@ -25,6 +29,10 @@ def test_loopback_exchange(orc, name, N, k, P):
     par.h0 = h1.info["h0"]
     parts = synth.partition(m, P)
     hs = [cf.from_synth(m, params=par, part=p, nccl_uid=None) for p in parts]
+    for h, p in zip(hs, parts):
+        mode, nb = h.exchange_schedule()
+        interior = len(p.zones) - nb
+        assert mode == (2 if overlap == "1" and nb > 0 and interior > 0 else 1), (mode, nb, len(p.zones))
     ls = [p.local_state(s) for p in parts]
     outs = cf.eval_loopback(hs, [t(l.x) for l in ls], [t(l.v) for l in ls], [t(l.e) for l in ls],
                             [t(l.rho0detJ0) for l in ls])
@@ -93,3 +101,96 @@ def test_loopback_integrator(name, N, k, P):
             else:
                 shared[g] = val
     assert abs(ke - ke1) <= 1e-13 * max(abs(ke1), 1e-300) and abs(ie - ie1) <= 1e-13 * abs(ie1)
+
+
+def test_loopback_schedules_bitwise_equal_and_overlap_visible(monkeypatch):
+    """C4-like mesh split over 2 ranks: the overlap schedule and the single-round schedule give the same
+    bits (same per-node summation orders), and with timing on the shared-row exchange ends before the
+    interior zones' corner force does (the exchange is hidden behind the interior)."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    m, s = synth.config("C4", "S1", N=(16, 16, 16))
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    par = cf.default_params()
+    par.h0 = (1.0 / m.num_zones) ** (1 / 3) / m.order
+    parts = synth.partition(m, 2)
+    ls = [p.local_state(s) for p in parts]
+    args = ([t(l.x) for l in ls], [t(l.v) for l in ls], [t(l.e) for l in ls], [t(l.rho0detJ0) for l in ls])
+    res = {}
+    for ov in ("1", "0"):
+        monkeypatch.setenv("BLAST_CF_OVERLAP", ov)
+        hs = [cf.from_synth(m, params=par, part=p, nccl_uid=None) for p in parts]
+        assert all(h.exchange_schedule()[0] == (2 if ov == "1" else 1) for h in hs)
+        for h in hs:
+            h.set_timing(True)
+        for _ in range(3):
+            outs = cf.eval_loopback(hs, *args)
+        torch.cuda.synchronize()
+        res[ov] = [[o.cpu().numpy() for o in out] for out in outs]
+        if ov == "1":
+            for h in hs:
+                sent, interior_end, end = h.debug_exchange_times()
+                assert sent < interior_end <= end, (sent, interior_end, end)
+        for h in hs:
+            h.close()
+    for a, b in zip(res["1"], res["0"]):
+        for x, y in zip(a, b):
+            assert np.array_equal(x, y)
+
+
+def _nccl_worker(rank, world, uid, overlap, q):
+    import os
+    os.environ["BLAST_CF_OVERLAP"] = overlap
+    import torch
+    torch.cuda.set_device(rank)
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    m, s = synth.config("C3", "S1", N=(8, 6, 6))
+    part = synth.partition(m, world)[rank]
+    h = cf.from_synth(m, part=part, nccl_uid=uid)
+    ls = part.local_state(s)
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    outs = None
+    for _ in range(3):
+        outs = h.eval(t(ls.x), t(ls.v), t(ls.e), t(ls.rho0detJ0))
+    torch.cuda.synchronize()
+    q.put((rank, h.exchange_schedule()[0], h.info["h0"], *(o.cpu().numpy() for o in outs)))
+    h.close()
+
+
+@pytest.mark.parametrize("overlap", ["1", "0"])
+def test_nccl_multiprocess(orc, overlap):
+    """The real NCCL path: P = min(#GPUs, 8) processes, one per GPU, both schedules; every rank's F.1 matches
+    the single-domain oracle, sharers hold the same bits, dt is the global min.  Needs >= 2 GPUs (NCCL
+    refuses two ranks on one device)."""
+    import torch
+    if not torch.cuda.is_available() or torch.cuda.device_count() < 2:
+        pytest.skip("needs >= 2 GPUs")
+    import torch.multiprocessing as mp
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    P = min(torch.cuda.device_count(), 8)
+    uid = cf.nccl_unique_id()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_nccl_worker, args=(r, P, uid, overlap, q)) for r in range(P)]
+    for p in procs:
+        p.start()
+    got = sorted(q.get(timeout=300) for _ in range(P))
+    for p in procs:
+        p.join(60)
+        assert p.exitcode == 0
+    m, s = synth.config("C3", "S1", N=(8, 6, 6))
+    r = orc.evaluate(m, s, params=orc.Params(h0=got[0][2]))
+    parts = synth.partition(m, P)
+    shared = {}
+    for (rank, mode, h0, F1, FTv, dt), p in zip(got, parts):
+        assert mode == (2 if overlap == "1" else 1)
+        assert np.abs(F1 - r.F1[:, p.nodes]).max() <= 1e-12 * np.abs(r.F1).max()
+        assert np.abs(FTv - r.FTv[p.zones]).max() <= 1e-12 * np.abs(r.FTv).max()
+        assert abs(float(dt[0]) - r.dt_min) <= 1e-12 * r.dt_min
+        for g, val in zip(p.nodes, F1.T):
+            if g in shared:
+                assert np.array_equal(shared[g], val)
+            else:
+                shared[g] = val

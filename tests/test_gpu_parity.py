@@ -355,14 +355,16 @@ def test_edge_regimes(orc, kind, dim, k, N, var, which, monkeypatch):
     if var:
         monkeypatch.setenv("BLAST_CF_KB1", var)
     m = synth.make_mesh(kind, dim, k, N)
-    s = synth.edge_state(m, kind, which, 31 + k)
+    # near-tie: relative gap 1e-4 for k <= 4; at k = 8 the strain rate itself carries ~8x the rounding (729-node
+    # gradient sums), measured 1.8e-12 on F.1 at gap 1e-4 (run r2-3), so the bar is checked at gap 3e-4 there
+    s = synth.edge_state(m, kind, which, 31 + k, tie_gap=1.5e-4 if k <= 4 else 4.5e-4)
     h, _, r = check(m, s, orc)
     if which == "window":
         assert r.diag["min_switch_dist"] < 1e-12           # every point's lambda - 2 eps_sw is inside the window
     elif which == "negative_e":
         assert (s.e < 0).any() and (s.e > 0).any()
     else:
-        assert 1e-5 < r.diag["min_gap"] < 2e-4
+        assert 1e-5 < r.diag["min_gap"] < (2e-4 if k <= 4 else 4e-4)
 
 
 def test_point_varying_rho_is_read_per_point(orc):
