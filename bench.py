@@ -430,6 +430,8 @@ def run_ours(args):
                          "kernel": f"KB1 (fused corner force, variant {h.variant})",
                          "kernel_ms": kb1_ms, "kb2_ms": float(kb[1]), "exchange_ms": float(kb[2]),
                          "flops_per_zone": info["flops_per_zone"],
+                         "flop_model": "SURVEY §8(d4) F_sf (c_pt 500 3D / 200 2D)",
+                         "frac_round1_model": info["flops_per_zone_alg"] * Zl / (kb1_ms / 1e3) / 1e12 / FP64_PEAK_TFLOPS,
                          "peak_note": "FP64 ALU: 148 SM x 64 FMA/clk x 2 x 1.965 GHz (measured DFMA 34.2 / DMMA 37.1 TF)",
                          "traffic_source": tsrc},
             "e2e": e2e,

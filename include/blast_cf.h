@@ -162,9 +162,10 @@ typedef struct {
   int64_t num_zones, num_nodes;
   double h0;                  /* the length scale in use */
   int32_t zones_per_cta, threads_per_cta, num_ctas, smem_bytes, regs_per_thread, local_bytes;
-  double flops_per_zone;      /* algorithmic FP64 flops per zone (DESIGN.md §5 model) */
+  double flops_per_zone;      /* algorithmic FP64 flops per zone: SURVEY §8(d4) F_sf */
   double alg_bytes;           /* algorithmic HBM bytes per eval */
   int32_t kernels_per_eval;   /* CUDA kernels launched by one eval */
+  double flops_per_zone_alg;  /* round 1's lower flop model (6 n^3 p last stage, c_pt 420 / 160), for comparison */
 } blast_cf_info;
 
 int blast_cf_get_info(const blast_cf *h, blast_cf_info *info);

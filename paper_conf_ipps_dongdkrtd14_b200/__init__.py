@@ -59,7 +59,7 @@ class Info(ctypes.Structure):
                 ("h0", ctypes.c_double), ("zones_per_cta", ctypes.c_int32), ("threads_per_cta", ctypes.c_int32),
                 ("num_ctas", ctypes.c_int32), ("smem_bytes", ctypes.c_int32), ("regs_per_thread", ctypes.c_int32),
                 ("local_bytes", ctypes.c_int32), ("flops_per_zone", ctypes.c_double), ("alg_bytes", ctypes.c_double),
-                ("kernels_per_eval", ctypes.c_int32)]
+                ("kernels_per_eval", ctypes.c_int32), ("flops_per_zone_alg", ctypes.c_double)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

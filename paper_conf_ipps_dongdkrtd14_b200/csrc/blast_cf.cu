@@ -24,6 +24,7 @@
 #include "kb1_v6.cuh"
 #include "kb1_v10.cuh"
 #include "kb1_v8.cuh"
+#include "kb1_v11.cuh"
 #include "kb1_p2d.cuh"
 #include "kb2_gather.cuh"
 #include "tables.h"
@@ -157,6 +158,16 @@ KB1Variant variant3v8() {
   using C = KB1V8Cfg<K>;
   return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v8<K, MINB>, (const void *)&kb1_v8_3d<K, MINB>, false, nullptr};
 }
+template <int K, int MINB>
+void launch3v11(const KB1Args &a, int grid, cudaStream_t s) {
+  using C = KB1V11Cfg<K>;
+  kb1_v11_3d<K, MINB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+}
+template <int K, int MINB>
+KB1Variant variant3v11() {
+  using C = KB1V11Cfg<K>;
+  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v11<K, MINB>, (const void *)&kb1_v11_3d<K, MINB>, true, nullptr};
+}
 template <int K, int ZPC, int MINB>
 KB1Variant variant3() {
   using C = KB1Cfg3<K, ZPC>;
@@ -199,8 +210,8 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
         break;
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
       case 6: add(variant3<6, 1, 2>(), "v1.z1m2"); add(variant3<6, 2, 1>(), "v1.z2"); break;
-      case 7: add(variant3v8<7, 1>(), "v8"); add(variant3<7, 1, 2>(), "v1.z1"); break;
-      case 8: add(variant3v8<8, 2>(), "v8"); add(variant3v8<8, 1>(), "v8.m1"); add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
+      case 7: add(variant3v8<7, 1>(), "v8"); add(variant3v11<7, 1>(), "v11"); add(variant3<7, 1, 2>(), "v1.z1"); break;
+      case 8: add(variant3v8<8, 2>(), "v8"); add(variant3v11<8, 2>(), "v11"); add(variant3v8<8, 1>(), "v8.m1"); add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
     }
   } else {
     switch (k) {
@@ -618,9 +629,19 @@ int check_async(blast_cf *h) {
   return BLAST_CF_OK;
 }
 
+// Algorithmic flops per zone: SURVEY §8(d4)'s F_sf verbatim (the contract's model):
+//   3D: 9 (4 n p^3 + 6 n^2 p^2 + 8 n^3 p) + 4 (n t^3 + n^2 t^2 + n^3 t) + 18 Nq + 500 Nq
+//   2D: 6 (4 n p^2 + 4 n^2 p) + 4 (n t^2 + n^2 t) + 8 Nq + 200 Nq
+// (FMA = 2 flops; c_pt = 500 / 200 per point with each div / sqrt / rsqrt = 1).  Round 1 used
+// a lower model (6 n^3 p in the last stage, c_pt 420 / 160): flops_per_zone_alg below, still reported.
 double flops_per_zone(int dim, int k) {
-  // sum-factorized contractions + counted pointwise flops (FMA = 2 flops; each
-  // div / sqrt / rsqrt / acos / cos = 1 flop).
+  const double n = 2 * k, p = k + 1, t = k;
+  if (dim == 3)
+    return 9.0 * (4 * n * p * p * p + 6 * n * n * p * p + 8 * n * n * n * p) + 4.0 * (n * t * t * t + n * n * t * t + n * n * n * t) +
+           18.0 * n * n * n + 500.0 * n * n * n;
+  return 6.0 * (4 * n * p * p + 4 * n * n * p) + 4.0 * (n * t * t + n * n * t) + 8.0 * n * n + 200.0 * n * n;
+}
+double flops_per_zone_alg(int dim, int k) {
   const double n = 2 * k, p = k + 1, t = k;
   if (dim == 3) {
     const double contr = 9.0 * (4 * n * p * p * p + 6 * n * n * p * p + 6 * n * n * n * p) +
@@ -1423,6 +1444,7 @@ int blast_cf_get_info(const blast_cf *h, blast_cf_info *info) {
   info->zones_per_cta = h->var.zpc; info->threads_per_cta = h->var.nth; info->num_ctas = h->ncta;
   info->smem_bytes = h->var.smem; info->regs_per_thread = h->regs; info->local_bytes = h->local_bytes;
   info->flops_per_zone = flops_per_zone(h->dim, h->k);
+  info->flops_per_zone_alg = flops_per_zone_alg(h->dim, h->k);
   // x, v read once, F.1 written once, e read, F^T v written, rho0|J0| read, dt
   info->alg_bytes = 8.0 * (3.0 * h->dim * h->nn + (double)h->Z * (2.0 * h->nt + h->nq)) + 8.0;
   info->kernels_per_eval = 2 + (h->xch ? blastcf::exchange_kernels(h->xch) : 0);

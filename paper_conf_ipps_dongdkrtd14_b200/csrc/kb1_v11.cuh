@@ -1,0 +1,371 @@
+// KB1 v11 — persistent 3D corner force for high orders (k = 7, 8; C5 is k = 8): kb1_v8.cuh's per-slab
+// stages, with the two costs ncu attributed to v8 (gpurun_out c5_v8 capture) removed:
+//   * the gather of every zone stalled all warps at the start of the CTA (13 % of the warp-stall samples:
+//     node ids -> coordinates, dependent DRAM loads).  v11 is persistent (2 CTAs per SM walk zones
+//     z = blockIdx.x + i * gridDim.x) and gathers zone i+1 by cp.async into sX / sE right after stage A of
+//     zone i's LAST slab (the only reader of sX / sE), so the copies fly under the remaining five stages
+//     of that slab; the next zone's node ids and e are prefetched into L2 at its first slab;
+//   * stage B^T ran on 3 of 8 warps (up to 288 DFMA per thread while 5 warps waited at the barrier):
+//     v11 splits every B^T item's a1 outputs over warps so all 8 warps work (at most 32 loads + 96 DFMA).
+// Mathematics, slab order, summation orders and outputs are those of v8 (eq (4)-(6); DESIGN.md
+// §1 rows a0-a5); J0^{-1} and gamma are double-buffered (the point stage of the last slab still reads
+// zone i's while zone i+1's arrive).
+#pragma once
+#include "kb1_v8.cuh"
+
+template <int K>
+struct V11Dims : V8Dims<K> {
+  using B = V8Dims<K>;
+  // O_J0 region grows from 10 to 20 doubles (two buffers of J0^{-1}[9] + gamma)
+  static constexpr int FIX = (B::O_J0 + 20 + 1) / 2 * 2;
+  static constexpr int OFF_FIX = B::TAB, OFF_A = OFF_FIX + FIX, OFF_B = OFF_A + (B::RA + 1) / 2 * 2;
+  static constexpr int OFF_RED = OFF_B + (B::RB + 1) / 2 * 2;
+  static constexpr int TOTAL = OFF_RED + 32;
+};
+
+template <int K>
+struct KB1V11Cfg {
+  using Dm = V11Dims<K>;
+  static constexpr int NTH = (Dm::NS + 31) / 32 * 32;
+  static constexpr int SMEM_BYTES = Dm::TOTAL * 8;
+};
+
+template <int K, int MINB>
+__global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1Args a) {
+  using Dm = V11Dims<K>;
+  constexpr int N = Dm::N, P = Dm::P, T = Dm::T, P2 = Dm::P2, NK = Dm::NK, NT = Dm::NT, NS = Dm::NS;
+  constexpr int T2 = Dm::T2, PP = Dm::PP, SR = Dm::SR;
+  constexpr int NTH = KB1V11Cfg<K>::NTH;
+  constexpr bool FILTER = NS % 32 == 0;   // every warp full of points: the dt filter's vote is legal
+  static_assert(NTH >= 192, "stage C^T: six warps of row items (k >= 7)");
+  static_assert(NTH >= 6 * 3 * P + T, "stage B: one item per thread");
+  static_assert(NTH >= 3 * P2, "stage A^T: one item per thread");
+  static_assert(P % 3 == 0 || P == 8, "stage B^T: a1 split in three parts of P/3 (k = 8) or two of 4 (k = 7)");
+  static_assert(3 * P <= 32, "stage B^T: one (c, a0) item per lane");
+  constexpr int NPART = P % 3 == 0 ? 3 : 2, PL = P / NPART;   // B^T: a1 parts per item
+  extern __shared__ double smem[];
+  double *sB = smem, *sG = sB + N * P, *sPhi = sG + N * P, *sW = sPhi + N * Dm::TS;
+  double *sF = smem + Dm::OFF_FIX;
+  double *sX = sF + Dm::O_X, *sE = sF + Dm::O_E, *sAF = sF + Dm::O_AF, *sAE = sF + Dm::O_AE, *sJ0b = sF + Dm::O_J0;
+  double *sA = smem + Dm::OFF_A, *sBr = smem + Dm::OFF_B, *sRed = smem + Dm::OFF_RED;
+
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int64_t Z = a.num_zones, nn = a.num_nodes, G = gridDim.x;
+  const int64_t nz = Z > blockIdx.x ? (Z - 1 - blockIdx.x) / G + 1 : 0;
+  auto zone_of = [&](int64_t i) { return (int64_t)blockIdx.x + i * G; };
+
+  // gather of zone i (cp.async; the caller commits / waits): X, V [6][NK], e [NT], J0^{-1} + gamma
+  auto gather = [&](int64_t i) {
+    const int64_t z = zone_of(i);
+    for (int r = tid; r < NK; r += NTH) {
+      const int64_t node = __ldg(a.zone_nodes + z * NK + r);
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        cp_async8(sX + c * NK + r, a.x + c * nn + node, true);
+        cp_async8(sX + (3 + c) * NK + r, a.v + c * nn + node, true);
+      }
+    }
+    for (int r = tid; r < NT; r += NTH) cp_async8(sE + r, a.e + z * NT + r, true);
+    if (tid < 10) cp_async8(sJ0b + (i & 1) * 10 + tid, tid < 9 ? a.J0inv + z * 9 + tid : a.zone_gamma + z, true);
+  };
+
+  // ---- tables, zone 0's gather, accumulators ------------------------------------------------------
+  for (int i = tid; i < 2 * N * P + N * T + N; i += NTH) {   // B, G; Phi into rows of TS; W
+    const double t = __ldg(a.tab + i);
+    if (i < 2 * N * P) smem[i] = t;
+    else if (i < 2 * N * P + N * T) sPhi[((i - 2 * N * P) / T) * Dm::TS + (i - 2 * N * P) % T] = t;
+    else sW[i - 2 * N * P - N * T] = t;
+  }
+  for (int r = tid; r < 3 * NK; r += NTH) sAF[r] = 0.0;
+  for (int r = tid; r < NT; r += NTH) sAE[r] = 0.0;
+  if (tid == 0) sRed[8] = 0.0;   // dt filter: the CTA's best exact inverse dt
+  if (nz > 0) gather(0);
+  cp_async_commit();
+  cp_async_wait<0>();
+  __syncthreads();
+
+  const int q0 = tid % N, q1 = tid / N;
+  const bool has_point = tid < NS;
+  double dtmin = __longlong_as_double(0x7ff0000000000000LL);
+  bool bad = false;
+
+#pragma unroll 1
+  for (int64_t zi = 0; zi < nz; ++zi) {
+    const int64_t z = zone_of(zi);
+    const double *sJ0 = sJ0b + (zi & 1) * 10;
+    const bool more = zi + 1 < nz;
+#pragma unroll 1
+    for (int q2 = 0; q2 < N; ++q2) {
+      const int o = a.zero * (q2 + 1);   // 0, but loop-variant and uniform: the table loads stay here
+      if (has_point)
+        asm volatile("prefetch.global.L1 [%0];" ::"l"(a.rho0detJ0 + z * (int64_t)(N * NS) + (q2 * N + q1) * N + q0));
+      if (q2 == 0 && more) {   // the next zone's node ids and e into L2, 15 slabs ahead of their use
+        const int64_t z1 = zone_of(zi + 1);
+        if (tid * 32 < NK) asm volatile("prefetch.global.L2 [%0];" ::"l"(a.zone_nodes + z1 * NK + tid * 32));
+        if (tid * 16 < NT) asm volatile("prefetch.global.L2 [%0];" ::"l"(a.e + z1 * NT + tid * 16));
+      }
+      // ---- stage A: a2 -> q2 (TB, TG of the 6 fields; TE) -------------------------------------------
+      {
+        const CTZ<K> C{o};
+#pragma unroll
+        for (int rd = 0; rd < (6 * P2 + T2 + NTH - 1) / NTH; ++rd) {
+          const int r = tid + rd * NTH;
+          if (r < 6 * P2) {
+            const int f = r / P2, rr = r - f * P2;
+            double tb = 0.0, tg = 0.0;
+#pragma unroll
+            for (int a2 = 0; a2 < P; ++a2) {
+              const double xv = sX[f * NK + a2 * P2 + rr];
+              tb = fma(C.B(q2, a2), xv, tb);
+              tg = fma(C.G(q2, a2), xv, tg);
+            }
+            sA[f * P2 + rr] = tb;
+            sA[6 * P2 + f * P2 + rr] = tg;
+          } else if (r < 6 * P2 + T2) {
+            const int jj = r - 6 * P2;
+            double te = 0.0;
+#pragma unroll
+            for (int j2 = 0; j2 < T; ++j2) te = fma(C.Phi(q2, j2), sE[j2 * T2 + jj], te);
+            sA[12 * P2 + jj] = te;
+          }
+        }
+      }
+      __syncthreads();
+      // last slab: sX / sE are dead -> gather the next zone under the remaining stages of this slab
+      if (q2 == N - 1 && more) {
+        gather(zi + 1);
+        cp_async_commit();
+      }
+      // ---- stage B: a1 -> q1; item (f, m, a0) produces U[f][m][q1 = 0..N-1][a0] --------------------
+      {
+        const CTZ<K> C{2 * o};
+        const int r = tid;
+        if (r < 18 * P) {
+          const int fm = r / P, a0 = r - fm * P, f = fm / 3, m = fm - f * 3;
+          const double *src = sA + (m == 2 ? 6 * P2 : 0) + f * P2 + a0;   // TG for m = 2, else TB
+          double tv[P];
+#pragma unroll
+          for (int a1 = 0; a1 < P; ++a1) tv[a1] = src[a1 * P];
+          double *U = sBr + fm * N * PP + a0;
+          if (m == 1) {
+#pragma unroll
+            for (int qq1 = 0; qq1 < N; ++qq1) {
+              double u = 0.0;
+#pragma unroll
+              for (int a1 = 0; a1 < P; ++a1) u = fma(C.G(qq1, a1), tv[a1], u);
+              U[qq1 * PP] = u;
+            }
+          } else {
+#pragma unroll
+            for (int qq1 = 0; qq1 < N; ++qq1) {
+              double u = 0.0;
+#pragma unroll
+              for (int a1 = 0; a1 < P; ++a1) u = fma(C.B(qq1, a1), tv[a1], u);
+              U[qq1 * PP] = u;
+            }
+          }
+          if (P < PP) {   // zero pad of the 16-byte pairs (read by stage C's paired loads, coefficient 0)
+#pragma unroll
+            for (int qq1 = 0; qq1 < N; ++qq1)
+              if (a0 == P - 1) U[qq1 * PP + 1] = 0.0;
+          }
+        } else if (r < 18 * P + T) {
+          const int j0 = r - 18 * P;
+          double tv[T];
+#pragma unroll
+          for (int j1 = 0; j1 < T; ++j1) tv[j1] = sA[12 * P2 + j1 * T + j0];
+#pragma unroll
+          for (int qq1 = 0; qq1 < N; ++qq1) {
+            double u = 0.0;
+#pragma unroll
+            for (int j1 = 0; j1 < T; ++j1) u = fma(C.Phi(qq1, j1), tv[j1], u);
+            sBr[18 * N * PP + qq1 * T + j0] = u;
+          }
+        }
+      }
+      __syncthreads();
+      // ---- stage C (a0 -> q0) + point evaluation ----------------------------------------------------
+      if (has_point) {
+        double g18[18];
+#pragma unroll
+        for (int i = 0; i < 18; ++i) g18[i] = 0.0;
+#pragma unroll
+        for (int pa = 0; pa < PP / 2; ++pa) {
+          const int a0 = 2 * pa;
+          const double b0 = sB[q0 * P + a0], g0 = sG[q0 * P + a0];
+          const double b1 = a0 + 1 < P ? sB[q0 * P + a0 + 1] : 0.0, g1 = a0 + 1 < P ? sG[q0 * P + a0 + 1] : 0.0;
+#pragma unroll
+          for (int fm = 0; fm < 18; ++fm) {
+            double u0, u1;
+            lds_f64x2(sBr + (fm * N + q1) * PP + a0, u0, u1);
+            const bool dx = fm % 3 == 0;
+            g18[fm] = fma(dx ? g0 : b0, u0, g18[fm]);
+            g18[fm] = fma(dx ? g1 : b1, u1, g18[fm]);
+          }
+        }
+        double eq = 0.0;
+#pragma unroll
+        for (int j0 = 0; j0 < T; ++j0) eq = fma(sPhi[q0 * Dm::TS + j0], sBr[18 * N * PP + q1 * T + j0], eq);
+        double Jm[3][3], Gv[3][3];
+#pragma unroll
+        for (int c = 0; c < 3; ++c)
+#pragma unroll
+          for (int d = 0; d < 3; ++d) { Jm[c][d] = g18[c * 3 + d]; Gv[c][d] = g18[9 + c * 3 + d]; }
+        const int q = (q2 * N + q1) * N + q0;
+        const double R = __ldg(a.rho0detJ0 + z * (int64_t)(N * NS) + q);
+        const double alpha = sW[q0] * sW[q1] * sW[q2];
+        PointOut<3> pt;
+        if (FILTER) {
+          const double best = sRed[8];
+          point_eval3<true>(Jm, Gv, eq, R, alpha, sJ0[9], sJ0, a.ph, pt, best);
+          double mi = pt.inv;
+#pragma unroll
+          for (int s = 16; s > 0; s >>= 1) mi = fmax(mi, __shfl_xor_sync(0xffffffffu, mi, s));
+          if (lane == 0 && mi > best)
+            atomicMax(reinterpret_cast<unsigned long long *>(sRed + 8), (unsigned long long)__double_as_longlong(mi));
+        } else {
+          point_eval3(Jm, Gv, eq, R, alpha, sJ0[9], sJ0, a.ph, pt);
+        }
+        double *S = sA + q1 * SR + q0;
+#pragma unroll
+        for (int cd = 0; cd < 9; ++cd) S[cd * N * SR] = pt.S[cd / 3][cd % 3];
+        S[9 * N * SR] = pt.P;
+        if (a.Sq != nullptr) {
+#pragma unroll
+          for (int cd = 0; cd < 9; ++cd) a.Sq[(z * (int64_t)(N * NS) + q) * 9 + cd] = pt.S[cd / 3][cd % 3];
+        }
+        dtmin = fmin(dtmin, pt.dt);
+        bad |= pt.bad;
+      }
+      __syncthreads();
+      // ---- stage C^T: q0 -> a0; warps 0-1: d = 0 components (G), 2-4: d != 0 (B), 5: Pq (Phi) -------
+      {
+        const CTZ<K> C{3 * o};
+        const int grp = warp < 2 ? 0 : warp < 5 ? 1 : warp < 6 ? 2 : 3;
+        const int li = (warp - (grp == 0 ? 0 : grp == 1 ? 2 : 5)) * 32 + lane;   // index inside the group
+        const int cdi = li / N, qq1 = li - cdi * N;
+        int cd = -1;
+        if (grp == 0 && cdi < 3) cd = cdi * 3;                         // 0, 3, 6
+        if (grp == 1 && cdi < 6) cd = (cdi / 2) * 3 + 1 + (cdi & 1);   // 1, 2, 4, 5, 7, 8
+        if (grp == 2 && cdi < 1) cd = 9;
+        if (cd >= 0 && qq1 < N) {
+          double sv[N];
+          const double *row = sA + (cd * N + qq1) * SR;
+#pragma unroll
+          for (int pq = 0; pq < N / 2; ++pq) lds_f64x2(row + 2 * pq, sv[2 * pq], sv[2 * pq + 1]);
+          if (grp == 0) {
+#pragma unroll
+            for (int a0 = 0; a0 < P; ++a0) {
+              double y = 0.0;
+#pragma unroll
+              for (int qq0 = 0; qq0 < N; ++qq0) y = fma(C.G(qq0, a0), sv[qq0], y);
+              sBr[(cd * N + qq1) * P + a0] = y;
+            }
+          } else if (grp == 1) {
+#pragma unroll
+            for (int a0 = 0; a0 < P; ++a0) {
+              double y = 0.0;
+#pragma unroll
+              for (int qq0 = 0; qq0 < N; ++qq0) y = fma(C.B(qq0, a0), sv[qq0], y);
+              sBr[(cd * N + qq1) * P + a0] = y;
+            }
+          } else {
+#pragma unroll
+            for (int j0 = 0; j0 < T; ++j0) {
+              double y = 0.0;
+#pragma unroll
+              for (int qq0 = 0; qq0 < N; ++qq0) y = fma(C.Phi(qq0, j0), sv[qq0], y);
+              sBr[9 * N * P + j0 * N + qq1] = y;
+            }
+          }
+        }
+      }
+      __syncthreads();
+      // ---- stage B^T: q1 -> a1 on all 8 warps: warps 0..NPART-1 ZB items (c, a0) for a1 part = warp,
+      //      the next NPART warps ZG items, the rest ZE items (j0) for j1 halves ------------------------
+      {
+        const CTZ<K> C{4 * o};
+        if (warp < NPART) {
+          if (lane < 3 * P) {
+            const int c = lane / P, a0 = lane - c * P, p0 = warp * PL;
+            const double *y0 = sBr + ((c * 3 + 0) * N) * P + a0, *y1 = sBr + ((c * 3 + 1) * N) * P + a0;
+            double v0[N], v1[N];
+#pragma unroll
+            for (int qq1 = 0; qq1 < N; ++qq1) { v0[qq1] = y0[qq1 * P]; v1[qq1] = y1[qq1 * P]; }
+#pragma unroll
+            for (int k1 = 0; k1 < PL; ++k1) {
+              double s = 0.0;
+#pragma unroll
+              for (int qq1 = 0; qq1 < N; ++qq1) {
+                s = fma(C.B(qq1, p0 + k1), v0[qq1], s);
+                s = fma(C.G(qq1, p0 + k1), v1[qq1], s);
+              }
+              sA[c * P2 + (p0 + k1) * P + a0] = s;
+            }
+          }
+        } else if (warp < 2 * NPART) {
+          if (lane < 3 * P) {
+            const int c = lane / P, a0 = lane - c * P, p0 = (warp - NPART) * PL;
+            const double *y2 = sBr + ((c * 3 + 2) * N) * P + a0;
+            double v2[N];
+#pragma unroll
+            for (int qq1 = 0; qq1 < N; ++qq1) v2[qq1] = y2[qq1 * P];
+#pragma unroll
+            for (int k1 = 0; k1 < PL; ++k1) {
+              double s = 0.0;
+#pragma unroll
+              for (int qq1 = 0; qq1 < N; ++qq1) s = fma(C.B(qq1, p0 + k1), v2[qq1], s);
+              sA[3 * P2 + c * P2 + (p0 + k1) * P + a0] = s;
+            }
+          }
+        } else {
+          constexpr int NEW = NTH / 32 - 2 * NPART;   // warps for the ZE items
+          constexpr int JL = (T + NEW - 1) / NEW;
+          const int j10 = (warp - 2 * NPART) * JL;
+          if (lane < T) {
+            const int j0 = lane;
+            double ve[N];
+#pragma unroll
+            for (int qq1 = 0; qq1 < N; ++qq1) ve[qq1] = sBr[9 * N * P + j0 * N + qq1];
+#pragma unroll
+            for (int k1 = 0; k1 < JL; ++k1) {
+              if (j10 + k1 < T) {
+                double s = 0.0;
+#pragma unroll
+                for (int qq1 = 0; qq1 < N; ++qq1) s = fma(C.Phi(qq1, j10 + k1), ve[qq1], s);
+                sA[6 * P2 + (j10 + k1) * T + j0] = s;
+              }
+            }
+          }
+        }
+      }
+      __syncthreads();
+      // ---- stage A^T: accumulate q2 -> a2; item (c, a1 a0) owns 9 accumulators, e items on the top -
+      {
+        const CTZ<K> C{5 * o};
+        if (tid < 3 * P2) {
+          const int c = tid / P2, rr = tid - c * P2;
+          const double zb = sA[c * P2 + rr], zg = sA[3 * P2 + c * P2 + rr];
+          double *acc = sAF + c * NK + rr;
+#pragma unroll
+          for (int a2 = 0; a2 < P; ++a2) acc[a2 * P2] = fma(C.B(q2, a2), zb, fma(C.G(q2, a2), zg, acc[a2 * P2]));
+        }
+        if (tid >= NTH - T2) {
+          const int jj = tid - (NTH - T2);
+          const double ze = sA[6 * P2 + jj];
+#pragma unroll
+          for (int j2 = 0; j2 < T; ++j2) sAE[j2 * T2 + jj] = fma(C.Phi(q2, j2), ze, sAE[j2 * T2 + jj]);
+        }
+      }
+      __syncthreads();   // region A (Z) is overwritten by the next slab's stage A
+    }
+    // ---- zone outputs; accumulators cleared for the next zone (same thread <-> entry mapping) -------
+    for (int i = tid; i < 3 * NK; i += NTH) { a.Fz1[z * 3 * NK + i] = sAF[i]; sAF[i] = 0.0; }
+    for (int i = tid; i < NT; i += NTH) { a.FTv[z * NT + i] = sAE[i]; sAE[i] = 0.0; }
+    cp_async_wait<0>();   // the next zone's X, V, e, J0^{-1} (issued in the last slab)
+    __syncthreads();
+  }
+  if (bad) dtmin = 0.0;
+  const double m = block_min(dtmin, sRed);
+  if (tid == 0) a.cta_dt[blockIdx.x] = m;
+}

@@ -63,8 +63,23 @@ def _worker(rank, world, port, name, N, k, q):
             for code in src[sptr[u]:sptr[u + 1]]:
                 acc += send[code] if code >= 0 else recv[-code - 1]
             F1[:, node] = acc
-        dt = torch.tensor([r.dt_min], dtype=torch.float64)
-        dist.all_reduce(dt, op=dist.ReduceOp.MIN)
+        # global min dt, as the library's single-round schedule does it: every rank's dt travels with its F.1
+        # rows to every neighbour (in these block partitions every rank neighbours every other, which the
+        # library checks before it drops the allreduce)
+        assert len(part.nbr_rank) == world - 1
+        mine = torch.tensor([r.dt_min], dtype=torch.float64)
+        got = []
+        for q_rank in part.nbr_rank:
+            t_in = torch.zeros(1, dtype=torch.float64)
+            a_ = dist.isend(mine.clone(), int(q_rank))
+            b_ = dist.irecv(t_in, int(q_rank))
+            a_.wait()
+            b_.wait()
+            got.append(float(t_in[0]))
+        dt = torch.tensor([min([r.dt_min] + got)], dtype=torch.float64)
+        ref_dt = torch.tensor([r.dt_min], dtype=torch.float64)
+        dist.all_reduce(ref_dt, op=dist.ReduceOp.MIN)   # the overlap schedule's allreduce gives the same value
+        assert float(ref_dt[0]) == float(dt[0])
         # --- checks against the single-domain oracle ---
         g = oracle.evaluate(mesh, st, params=par)
         ref = g.F1[:, part.nodes]
