@@ -205,7 +205,8 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
       case 4:
         // (round 2: the superseded generations v10 (runtime switches), v10.wu, v6, v5, v4.m0/m1, v3.z1 that never
         //  won the autotuner are no longer instantiated; DESIGN.md §10 keeps their measurements)
-        add(variant3v10<4, 0, 0, 0, 3>(), "v10.w"); add(variant3v10<4, 0, 0, 0, 2>(), "v10.v"); add(variant3v5<4, 0, 1>(), "v5.r1");
+        add(variant3v10<4, 0, 0, 0, 3>(), "v10.w");
+        add(variant3v10<4, 0, 0, 0, 2>(), "v10.v"); add(variant3v5<4, 0, 1>(), "v5.r1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;

@@ -89,6 +89,8 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   using Cfg = KB1V5Cfg<K, MODE>;
   constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4, PWG = OPT & 8, V16 = OPT & 16;
   constexpr bool NOXV = OPT & 32;   // timing diagnostic only (wrong results): no x / v gather
+  constexpr bool CLK = !(OPT & 4096);   // per-zone clock64 accounting (BLAST_CF_PROFILE); bit 12 compiles it out
+  constexpr int EIG = (OPT & 8192) ? 1 : 0;   // bit 13: branchy smallest eigenpair (pointwise.cuh sym3_min_eig)
   constexpr bool SPREAD = OPT & 64;   // the 6 P^3 node-field copies spread over all contraction threads
   static_assert(!V16 || (Dm::T3 % 2 == 0 && Dm::N3 % 2 == 0 && Dm::XE_E % 2 == 0 && (Dm::OFF_XE + Dm::XE_E) % 2 == 0 &&
                          (Dm::OFF_UV + Dm::O_R) % 2 == 0 && Dm::UVBUF % 2 == 0), "16-byte copies need 16-byte alignment");
@@ -539,8 +541,8 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     PointOut<3> oa, ob;
     const double best = sRed[8];   // largest exact inverse dt found so far by this CTA (dt filter)
     if (VMODE == 3 && a.ph.use_visc && a.ph.use_vort) {   // both points one straight-line block, one vote
-      point_eval3<2, 1>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best);
-      point_eval3<2, 1>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best);
+      point_eval3<2, 1, EIG>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best);
+      point_eval3<2, 1, EIG>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best);
       if (__any_sync(0xffffffffu, oa.cand || ob.cand)) {   // J is still in the JS buffer (S is written below)
         double Jr[3][3];
 #pragma unroll
@@ -612,7 +614,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     long long t_work = 0;
     int itc = 2;
     for (int64_t i = 0; i <= nz; ++i, ++itc) {
-      const long long t0 = clock64();
+      const long long t0 = CLK ? clock64() : 0;
       auto issue = [&] {
         kw_issue(i + 1);
         kw_load_id(i + 2);
@@ -634,7 +636,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       if (i + 1 < nz && DIAG != 1)
         kw_forward(sUV + ((i + 1) & 1) * Dm::UVBUF, sJS + ((i + 1) & 1) * Dm::JSBUF, sJ + ((i + 1) & 1) * 10, zc + a.zero,
                    PWG ? sXEb[(i + 1) & 1] : sXE);
-      t_work += clock64() - t0;
+      if (CLK) t_work += clock64() - t0;
       __syncthreads();
       kstamp(11);
     }
@@ -686,9 +688,9 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     cp_async_commit();
   }
   __syncthreads();
-  long long t_work = 0, t_all = clock64();
+  long long t_work = 0, t_all = CLK ? clock64() : 0;
   for (int64_t i = 0; i <= nz; ++i) {
-    const long long t0 = clock64();
+    const long long t0 = CLK ? clock64() : 0;
     if (i < nz && tid < TPZ && DIAG != 2)
       pw_point(sUV + (i & 1) * Dm::UVBUF, sJ + (i & 1) * 10, sJS + (i & 1) * Dm::JSBUF, zone_of(i));
     if (PWG) {   // zone i's points are done: issue zone i+2 (its XE and R slots were last read for zone i)
@@ -697,7 +699,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       pw_load_id(i + 3);
       cp_async_commit();
     }
-    t_work += clock64() - t0;
+    if (CLK) t_work += clock64() - t0;
     __syncthreads();
   }
   if (PWG) cp_async_wait<0>();
