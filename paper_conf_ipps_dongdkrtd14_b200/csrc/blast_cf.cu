@@ -567,6 +567,8 @@ struct blast_cf {
     int nch = 0;                             // zone chunks (1 = no pipelining)
     int64_t z0[MAXC + 1] = {};               // chunk c = zones [z0[c], z0[c+1])
     int64_t hi[MAXC] = {};                   // max node id over the zones of chunks 0..c (prefix max)
+    int64_t lo[MAXC + 1] = {};               // min node id over the zones of chunks c..nch-1 (suffix min; lo[nch] = nn):
+                                             // F.1 of nodes below lo[c+1] is final once chunks 0..c are done
     int grid[MAXC] = {}, off[MAXC] = {}, nslots = 0;   // KB1 grid and per-CTA dt slots of each chunk
     double *d_ctadt = nullptr;
     cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
@@ -910,13 +912,18 @@ static int comm_sms() {
   return e ? std::max(0, atoi(e)) : 4;
 }
 
-static void launch_kb2(const blast_cf *h, double *F1, const double *cta_dt, int ncta, double *dt, cudaStream_t st) {
+// KB2 on nodes [n0, n1) (default: all); dt != nullptr: its last block also reduces the per-CTA dt slots
+static void launch_kb2(const blast_cf *h, double *F1, const double *cta_dt, int ncta, double *dt, cudaStream_t st,
+                       int64_t n0 = 0, int64_t n1 = -1) {
+  if (n1 < 0) n1 = h->nn;
   const int gthreads = 256;
-  const int64_t gblocks = std::max<int64_t>(1, (h->nn + gthreads - 1) / gthreads);
+  const int64_t gblocks = std::max<int64_t>(1, (n1 - n0 + gthreads - 1) / gthreads);
   if (h->dim == 3)
-    kb2_gather<3, 8><<<(unsigned)gblocks, gthreads, 0, st>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->nk, F1, cta_dt, ncta, dt);
+    kb2_gather<3, 8><<<(unsigned)gblocks, gthreads, 0, st>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, n0, n1, h->nk, F1, cta_dt,
+                                                             ncta, dt);
   else
-    kb2_gather<2, 4><<<(unsigned)gblocks, gthreads, 0, st>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->nk, F1, cta_dt, ncta, dt);
+    kb2_gather<2, 4><<<(unsigned)gblocks, gthreads, 0, st>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, n0, n1, h->nk, F1, cta_dt,
+                                                             ncta, dt);
 }
 
 static void launch_pack_gather(const blast_cf *h, cudaStream_t st) {
@@ -1140,6 +1147,12 @@ static int host_plan(blast_cf *h) {
     P.off[c] = P.nslots;
     P.nslots += g;
   }
+  P.lo[nch] = h->nn;
+  for (int c = nch - 1; c >= 0; --c) {
+    int64_t m = P.lo[c + 1];
+    for (size_t i = (size_t)P.z0[c] * h->nk; nch > 1 && i < (size_t)P.z0[c + 1] * h->nk; ++i) m = std::min<int64_t>(m, zn[i]);
+    P.lo[c] = m;
+  }
   cudaFree(P.d_ctadt);
   P.d_ctadt = nullptr;
   CUDA_TRY(cudaMalloc(&P.d_ctadt, std::max(P.nslots, 1) * sizeof(double)));
@@ -1218,6 +1231,7 @@ int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const doub
   a.ph.eps_sw = h->params.eps_switch; a.ph.inv_2eps = 0.5 / h->params.eps_switch; a.ph.h0 = h->h0; a.ph.k = (double)h->k;
   a.ph.use_visc = h->params.use_viscosity; a.ph.use_vort = h->params.use_vorticity;
   int64_t done = 0;   // nodes [0, done) of x and v are on their way
+  int64_t gathered = 0;   // nodes [0, gathered) of F.1 are gathered and on their way back
   for (int c = 0; c < P.nch; ++c) {
     const int64_t z0 = P.z0[c], zc = P.z0[c + 1] - z0, n1 = P.hi[c] + 1;
     if (n1 > done) {
@@ -1246,17 +1260,23 @@ int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const doub
     CUDA_TRY(cudaStreamWaitEvent(P.s_d2h, P.ev_kb1[c], 0));
     CUDA_TRY(cudaMemcpyAsync(out_FTv + z0 * h->nt, dT + z0 * h->nt, zc * h->nt * sizeof(double), cudaMemcpyDeviceToHost,
                              P.s_d2h));
+    // nodes below lo[c+1] touch no later chunk: gather them now and send their F.1 back while later chunks compute
+    const int64_t g1 = c + 1 < P.nch ? P.lo[c + 1] : gathered;
+    if (g1 > gathered) {
+      launch_kb2(h, dF, nullptr, 0, nullptr, h->stream, gathered, g1);
+      CUDA_TRY(cudaEventRecord(P.ev_kb1[c], h->stream));
+      CUDA_TRY(cudaStreamWaitEvent(P.s_d2h, P.ev_kb1[c], 0));
+      for (int d = 0; d < h->dim; ++d)
+        CUDA_TRY(cudaMemcpyAsync(out_Fdot1 + d * h->nn + gathered, dF + d * h->nn + gathered,
+                                 (g1 - gathered) * sizeof(double), cudaMemcpyDeviceToHost, P.s_d2h));
+      gathered = g1;
+    }
   }
-  // (nodes above hi[nch-1] belong to no zone: KB2 gives them F.1 = 0 without reading x or v)
-  const int gthreads = 256;
-  const int64_t gblocks = std::max<int64_t>(1, (h->nn + gthreads - 1) / gthreads);
-  if (h->dim == 3)
-    kb2_gather<3, 8><<<(unsigned)gblocks, gthreads, 0, h->stream>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->nk, dF,
-                                                                     P.d_ctadt, P.nslots, dd);
-  else
-    kb2_gather<2, 4><<<(unsigned)gblocks, gthreads, 0, h->stream>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nn, h->nk, dF,
-                                                                     P.d_ctadt, P.nslots, dd);
-  CUDA_TRY(cudaMemcpyAsync(out_Fdot1, dF, nx * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+  // the remaining nodes and the min dt (nodes above hi[nch-1] belong to no zone: KB2 gives them F.1 = 0)
+  launch_kb2(h, dF, P.d_ctadt, P.nslots, dd, h->stream, gathered, h->nn);
+  for (int d = 0; d < h->dim; ++d)
+    CUDA_TRY(cudaMemcpyAsync(out_Fdot1 + d * h->nn + gathered, dF + d * h->nn + gathered, (h->nn - gathered) * sizeof(double),
+                             cudaMemcpyDeviceToHost, h->stream));
   CUDA_TRY(cudaMemcpyAsync(out_dt_min, dd, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
   CUDA_TRY(cudaEventRecord(P.ev_d2h, P.s_d2h));
   CUDA_TRY(cudaStreamWaitEvent(h->stream, P.ev_d2h, 0));

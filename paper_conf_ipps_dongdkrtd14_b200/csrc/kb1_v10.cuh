@@ -610,7 +610,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     }
     kw_bar<NKW>();
     if (nz > 0 && DIAG != 1) kw_forward(sUV, sJS, sJ, a.zero, sXEb[0]);
-    __syncthreads();
+    cta_bar_div<Cfg::NTH>();
     long long t_work = 0;
     int itc = 2;
     for (int64_t i = 0; i <= nz; ++i, ++itc) {
@@ -637,7 +637,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
         kw_forward(sUV + ((i + 1) & 1) * Dm::UVBUF, sJS + ((i + 1) & 1) * Dm::JSBUF, sJ + ((i + 1) & 1) * 10, zc + a.zero,
                    PWG ? sXEb[(i + 1) & 1] : sXE);
       if (CLK) t_work += clock64() - t0;
-      __syncthreads();
+      cta_bar_div<Cfg::NTH>();
       kstamp(11);
     }
     if (a.prof != nullptr && tid == NPW) {
@@ -687,7 +687,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     pw_load_id(2);
     cp_async_commit();
   }
-  __syncthreads();
+  cta_bar_div<Cfg::NTH>();
   long long t_work = 0, t_all = CLK ? clock64() : 0;
   for (int64_t i = 0; i <= nz; ++i) {
     const long long t0 = CLK ? clock64() : 0;
@@ -700,7 +700,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       cp_async_commit();
     }
     if (CLK) t_work += clock64() - t0;
-    __syncthreads();
+    cta_bar_div<Cfg::NTH>();
   }
   if (PWG) cp_async_wait<0>();
   if (a.prof != nullptr && tid == 0) {

@@ -67,6 +67,12 @@ __device__ __forceinline__ int opaque_tid() {
 
 template <int NKW>
 __device__ __forceinline__ void kw_bar() { asm volatile("bar.sync 1, %0;\n" ::"n"(NKW) : "memory"); }
+// The CTA-wide barrier of the warp-specialized kernels, reached by the point warps and the contraction warps
+// at DIFFERENT instructions: the non-aligned barrier.sync with the explicit thread count (legal in divergent
+// code; __syncthreads() is barrier.sync.aligned, which requires every thread of the CTA at the same
+// instruction — compute-sanitizer synccheck flagged it, gpurun_out r02_sanitizer)
+template <int NT>
+__device__ __forceinline__ void cta_bar_div() { asm volatile("barrier.sync 0, %0;\n" ::"n"(NT) : "memory"); }
 
 template <int K, int MODE>
 __global__ void __launch_bounds__(KB1V4Cfg<K, MODE>::NTH, 1) kb1_v4_3d(const KB1Args a) {

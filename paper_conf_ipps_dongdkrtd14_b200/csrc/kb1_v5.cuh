@@ -554,7 +554,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v5_3d(const KB1
     cp_async_wait<0>();
     kw_bar<NKW>();
     if (nz > 0 && DIAG != 1) kw_forward(sUV, sJS, sJ);
-    __syncthreads();
+    cta_bar_div<Cfg::NTH>();
     long long t_work = 0;
     for (int64_t i = 0; i <= nz; ++i) {
       const long long t0 = clock64();
@@ -569,7 +569,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v5_3d(const KB1
       if (i + 1 < nz && DIAG != 1)
         kw_forward(sUV + ((i + 1) & 1) * Dm::UVBUF, sJS + ((i + 1) & 1) * Dm::JSBUF, sJ + ((i + 1) & 1) * 10);
       t_work += clock64() - t0;
-      __syncthreads();
+      cta_bar_div<Cfg::NTH>();
       kstamp(11);
     }
     if (a.prof != nullptr && tid == NPW) {
@@ -579,14 +579,14 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v5_3d(const KB1
     return;
   }
   asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;\n" ::"n"(Cfg::REG_PW));
-  __syncthreads();
+  cta_bar_div<Cfg::NTH>();
   long long t_work = 0, t_all = clock64();
   for (int64_t i = 0; i <= nz; ++i) {
     const long long t0 = clock64();
     if (i < nz && tid < TPZ && DIAG != 2)
       pw_point(sUV + (i & 1) * Dm::UVBUF, sJ + (i & 1) * 10, sJS + (i & 1) * Dm::JSBUF, zone_of(i));
     t_work += clock64() - t0;
-    __syncthreads();
+    cta_bar_div<Cfg::NTH>();
   }
   if (a.prof != nullptr && tid == 0) {
     a.prof[blockIdx.x * 16 + 0] = t_work;

@@ -8,13 +8,16 @@
 // (unstructured meshes) finish in a loop.
 #pragma once
 
+// Nodes [n0, n1) of num_nodes (the host entry gathers node ranges as their zones complete); the last block
+// also reduces the per-CTA dt slots when dt_out != nullptr.
 template <int DIM, int MAXE>
 __global__ void __launch_bounds__(256) kb2_gather(const double *__restrict__ Fz1, const int32_t *__restrict__ ptr,
-                                                  const int32_t *__restrict__ ent, int64_t num_nodes, int nk,
-                                                  double *__restrict__ out, const double *__restrict__ cta_dt,
-                                                  int num_cta, double *__restrict__ dt_out) {
+                                                  const int32_t *__restrict__ ent, int64_t num_nodes, int64_t n0,
+                                                  int64_t n1, int nk, double *__restrict__ out,
+                                                  const double *__restrict__ cta_dt, int num_cta,
+                                                  double *__restrict__ dt_out) {
   __shared__ double red[32];
-  if (blockIdx.x == gridDim.x - 1) {
+  if (dt_out != nullptr && blockIdx.x == gridDim.x - 1) {
     double m = __longlong_as_double(0x7ff0000000000000LL);
     for (int i = threadIdx.x; i < num_cta; i += blockDim.x) m = fmin(m, cta_dt[i]);
 #pragma unroll
@@ -28,8 +31,8 @@ __global__ void __launch_bounds__(256) kb2_gather(const double *__restrict__ Fz1
       if (threadIdx.x == 0) *dt_out = r;
     }
   }
-  const int64_t n = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (n >= num_nodes) return;
+  const int64_t n = n0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (n >= n1) return;
   const int b = __ldg(ptr + n), e = __ldg(ptr + n + 1);
   int o[MAXE];
 #pragma unroll

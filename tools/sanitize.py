@@ -1,0 +1,56 @@
+#!/usr/bin/env python
+"""One small corner-force evaluation (or integrator step) for compute-sanitizer.
+
+    compute-sanitizer --tool memcheck|racecheck|synccheck python tools/sanitize.py <case>
+cases: c4 (v10.w, 3D k=4, 40 zones), c5 (v11, 3D k=8, 4 zones), c5v8 (v8), c3 (v2.z1m12, 3D k=2),
+       c2 (p2d.z2m6, 2D k=4), integrator (2D k=3 RK2 step), host (pipelined host entry, 3D k=2 16^3)."""
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+CASES = {"c4": ("C4", (5, 4, 2), None, "v10.w"), "c5": ("C5", (2, 1, 2), None, "v11"), "c5v8": ("C5", (2, 1, 2), None, "v8"),
+         "c3": ("C3", (4, 4, 3), None, "v2.z1m12"), "c2": ("C2", (9, 7), None, "p2d.z2m6")}
+
+
+def main(case):
+    import torch
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    import synth
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    if case in CASES:
+        name, N, k, var = CASES[case]
+        os.environ["BLAST_CF_KB1"] = var
+        m, s = synth.config(name, "S1", N=N, k=k)
+        h = cf.from_synth(m)
+        assert h.variant == var, h.variant
+        for _ in range(2):
+            F1, FTv, dt = h.eval(t(s.x), t(s.v), t(s.e), t(s.rho0detJ0))
+        torch.cuda.synchronize()
+        print(case, var, "dt", float(dt.cpu()[0]), "|F1|", float(F1.abs().max()))
+    elif case == "integrator":
+        m = synth.make_mesh("triple", 2, 3, (7, 3))
+        s = synth.make_state(m, "triple", "S1", 1)
+        h = cf.from_synth(m)
+        rk = cf.RK2(h, s.rho0detJ0)
+        x, v, e = t(s.x), t(s.v), t(s.e)
+        d, it = rk.step(x, v, e, 1e-3)
+        torch.cuda.synchronize()
+        print(case, "dt_est", d, "cg", it)
+    elif case == "host":
+        m, s = synth.config("C3", "S1", N=(16, 16, 16))
+        h = cf.from_synth(m)
+        hx = [torch.from_numpy(np.ascontiguousarray(a)).pin_memory() for a in (s.x, s.v, s.e, s.rho0detJ0)]
+        o = h.eval_host(*hx)
+        h.set_rho0detJ0_host(hx[3])
+        o = h.eval_host(hx[0], hx[1], hx[2], None)
+        print(case, "dt", o[2][0])
+    else:
+        raise SystemExit(f"unknown case {case}")
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main(sys.argv[1]))
