@@ -158,15 +158,16 @@ KB1Variant variant3v8() {
   using C = KB1V8Cfg<K>;
   return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v8<K, MINB>, (const void *)&kb1_v8_3d<K, MINB>, false, nullptr};
 }
-template <int K, int MINB>
+template <int K, int MINB, int MB>
 void launch3v11(const KB1Args &a, int grid, cudaStream_t s) {
   using C = KB1V11Cfg<K>;
-  kb1_v11_3d<K, MINB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+  kb1_v11_3d<K, MINB, MB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
 }
-template <int K, int MINB>
+template <int K, int MINB, int MB = 0>
 KB1Variant variant3v11() {
   using C = KB1V11Cfg<K>;
-  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v11<K, MINB>, (const void *)&kb1_v11_3d<K, MINB>, true, nullptr};
+  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v11<K, MINB, MB>, (const void *)&kb1_v11_3d<K, MINB, MB>, true,
+                    nullptr};
 }
 template <int K, int ZPC, int MINB>
 KB1Variant variant3() {
@@ -212,7 +213,7 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
       case 6: add(variant3<6, 1, 2>(), "v1.z1m2"); add(variant3<6, 2, 1>(), "v1.z2"); break;
       case 7: add(variant3v8<7, 1>(), "v8"); add(variant3v11<7, 1>(), "v11"); add(variant3<7, 1, 2>(), "v1.z1"); break;
-      case 8: add(variant3v8<8, 2>(), "v8"); add(variant3v11<8, 2>(), "v11"); add(variant3v8<8, 1>(), "v8.m1"); add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
+      case 8: add(variant3v11<8, 2, 1>(), "v11.mb"); add(variant3v8<8, 2>(), "v8"); add(variant3v11<8, 2>(), "v11"); add(variant3v8<8, 1>(), "v8.m1"); add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
     }
   } else {
     switch (k) {

@@ -30,7 +30,11 @@ struct KB1V11Cfg {
   static constexpr int SMEM_BYTES = Dm::TOTAL * 8;
 };
 
-template <int K, int MINB>
+// MB = 1: stage B on DMMA (mma.sync m8n8k4 f64): U_X[q1][col] = sum_a1 X[q1][a1] In[a1][col] for the tables
+// X = B (columns: the TB and TG lines of the 6 fields, 108) and X = G (the TB lines, 54), K = P padded to a
+// multiple of 4, plus the e lines with Phi (K = T): 22 n-tiles of 8 columns over the 8 warps.  One DMMA does
+// 256 FMAs (the DFMA form issues an LDCU of the table coefficient next to every DFMA).
+template <int K, int MINB, int MB = 0>
 __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1Args a) {
   using Dm = V11Dims<K>;
   constexpr int N = Dm::N, P = Dm::P, T = Dm::T, P2 = Dm::P2, NK = Dm::NK, NT = Dm::NT, NS = Dm::NS;
@@ -137,7 +141,60 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
         cp_async_commit();
       }
       // ---- stage B: a1 -> q1; item (f, m, a0) produces U[f][m][q1 = 0..N-1][a0] --------------------
-      {
+      if (MB) {
+        static_assert(!MB || (N == 16 && NTH == 256), "DMMA stage B is written for k = 8 (two m-tiles of q1)");
+        constexpr int KSP = (P + 3) / 4, KST = (T + 3) / 4;       // k-steps of the B/G and Phi contractions
+        constexpr int NB = (108 + 7) / 8, NG = (54 + 7) / 8;      // n-tiles of the B-table and G-table columns
+        constexpr int NTILE = NB + NG + 1;                          // + one tile of the 8 e lines
+        const int lr = lane >> 2, lc = lane & 3;
+        for (int tl = warp; tl < NTILE; tl += NTH / 32) {
+          const int tab = tl < NB ? 0 : tl < NB + NG ? 1 : 2;      // 0: B, 1: G, 2: Phi (warp-uniform)
+          const int c0 = (tab == 0 ? tl : tab == 1 ? tl - NB : 0) * 8;
+          const double *X = tab == 0 ? sB : tab == 1 ? sG : sPhi;
+          const int ldx = tab == 2 ? Dm::TS : P, kx = tab == 2 ? T : P, ncol = tab == 0 ? 108 : tab == 1 ? 54 : T;
+          // the column this lane feeds (B operand) and the two it receives (D operand): col -> source line
+          auto line_src = [&](int col) -> const double * {   // In[a1][col] = line_src(col)[a1 * stride]
+            if (tab == 2) return sA + 12 * P2 + col;                                      // TE[j1][j0 = col]
+            const int f = (col % 54) / P, a0 = col % P;
+            return sA + ((tab == 0 && col >= 54) ? 6 * P2 : 0) + f * P2 + a0;           // TG (B lines >= 54) or TB
+          };
+          const int bcol = c0 + lr;
+          const double *bsrc = bcol < ncol ? line_src(bcol) : nullptr;
+          const int bstride = tab == 2 ? T : P;
+          double d[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
+#pragma unroll
+          for (int ks = 0; ks < KSP; ++ks) {
+            if (tab == 2 && ks >= KST) break;
+            const int kk = 4 * ks + lc;
+            const double b = (bsrc != nullptr && kk < kx) ? bsrc[kk * bstride] : 0.0;
+#pragma unroll
+            for (int mt = 0; mt < 2; ++mt) {
+              const int row = 8 * mt + lr;
+              const double af = kk < kx ? X[row * ldx + kk] : 0.0;
+              dmma(d[mt][0], d[mt][1], af, b);
+            }
+          }
+#pragma unroll
+          for (int i = 0; i < 2; ++i) {
+            const int col = c0 + 2 * lc + i;
+            if (col < ncol) {
+#pragma unroll
+              for (int mt = 0; mt < 2; ++mt) {
+                const int q1o = 8 * mt + lr;
+                if (tab == 2) {
+                  sBr[18 * N * PP + q1o * T + col] = d[mt][i];
+                } else {
+                  const int f = (col % 54) / P, a0 = col % P;
+                  const int fm = 3 * f + (tab == 1 ? 1 : col >= 54 ? 2 : 0);
+                  double *U = sBr + fm * N * PP + q1o * PP + a0;
+                  U[0] = d[mt][i];
+                  if (P < PP && a0 == P - 1) U[1] = 0.0;   // zero pad of the 16-byte pairs
+                }
+              }
+            }
+          }
+        }
+      } else {
         const CTZ<K> C{2 * o};
         const int r = tid;
         if (r < 18 * P) {
