@@ -123,8 +123,14 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
               tb = fma(C.B(q2, a2), xv, tb);
               tg = fma(C.G(q2, a2), xv, tg);
             }
-            sA[f * P2 + rr] = tb;
-            sA[6 * P2 + f * P2 + rr] = tg;
+            if (MB) {   // [a1][108] lines: TB of the 6 fields (f, a0) in columns 0..53, TG in 54..107
+              const int a1 = rr / P, a0 = rr - a1 * P;
+              sA[a1 * 108 + f * P + a0] = tb;
+              sA[a1 * 108 + 54 + f * P + a0] = tg;
+            } else {
+              sA[f * P2 + rr] = tb;
+              sA[6 * P2 + f * P2 + rr] = tg;
+            }
           } else if (r < 6 * P2 + T2) {
             const int jj = r - 6 * P2;
             double te = 0.0;
@@ -147,48 +153,53 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
         constexpr int NB = (108 + 7) / 8, NG = (54 + 7) / 8;      // n-tiles of the B-table and G-table columns
         constexpr int NTILE = NB + NG + 1;                          // + one tile of the 8 e lines
         const int lr = lane >> 2, lc = lane & 3;
-        for (int tl = warp; tl < NTILE; tl += NTH / 32) {
-          const int tab = tl < NB ? 0 : tl < NB + NG ? 1 : 2;      // 0: B, 1: G, 2: Phi (warp-uniform)
-          const int c0 = (tab == 0 ? tl : tab == 1 ? tl - NB : 0) * 8;
-          const double *X = tab == 0 ? sB : tab == 1 ? sG : sPhi;
-          const int ldx = tab == 2 ? Dm::TS : P, kx = tab == 2 ? T : P, ncol = tab == 0 ? 108 : tab == 1 ? 54 : T;
-          // the column this lane feeds (B operand) and the two it receives (D operand): col -> source line
-          auto line_src = [&](int col) -> const double * {   // In[a1][col] = line_src(col)[a1 * stride]
-            if (tab == 2) return sA + 12 * P2 + col;                                      // TE[j1][j0 = col]
-            const int f = (col % 54) / P, a0 = col % P;
-            return sA + ((tab == 0 && col >= 54) ? 6 * P2 : 0) + f * P2 + a0;           // TG (B lines >= 54) or TB
-          };
-          const int bcol = c0 + lr;
-          const double *bsrc = bcol < ncol ? line_src(bcol) : nullptr;
-          const int bstride = tab == 2 ? T : P;
-          double d[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
+        static_assert(!MB || 6 * P == 54, "the [a1][108] T layout");
 #pragma unroll
-          for (int ks = 0; ks < KSP; ++ks) {
-            if (tab == 2 && ks >= KST) break;
-            const int kk = 4 * ks + lc;
-            const double b = (bsrc != nullptr && kk < kx) ? bsrc[kk * bstride] : 0.0;
+        for (int rr = 0; rr < (NTILE + NTH / 32 - 1) / (NTH / 32); ++rr) {
+          const int tl = warp + rr * (NTH / 32);
+          if (tl < NTILE) {
+            const int tab = tl < NB ? 0 : tl < NB + NG ? 1 : 2;      // 0: B, 1: G, 2: Phi (warp-uniform)
+            const int c0 = (tab == 0 ? tl : tab == 1 ? tl - NB : 0) * 8;
+            const double *X = tab == 0 ? sB : tab == 1 ? sG : sPhi;
+            const int ldx = tab == 2 ? Dm::TS : P, kx = tab == 2 ? T : P, ncol = tab == 0 ? 108 : tab == 1 ? 54 : T;
+            // B operand In[a1][col]: the [a1][108] T lines (B and G tables) or TE[j1][j0] (Phi): linear in col
+            const int bcol = c0 + lr;
+            const double *bsrc = (tab == 2 ? sA + 12 * P2 : sA) + bcol;
+            const int bstride = tab == 2 ? T : 108;
+            const bool bok = bcol < ncol;
+            double d[2][2] = {{0.0, 0.0}, {0.0, 0.0}};
 #pragma unroll
-            for (int mt = 0; mt < 2; ++mt) {
-              const int row = 8 * mt + lr;
-              const double af = kk < kx ? X[row * ldx + kk] : 0.0;
-              dmma(d[mt][0], d[mt][1], af, b);
+            for (int ks = 0; ks < KSP; ++ks) {
+              const int kk = 4 * ks + lc;
+              if (tab != 2 || ks < KST) {
+                const double b = (bok && kk < kx) ? bsrc[kk * bstride] : 0.0;
+#pragma unroll
+                for (int mt = 0; mt < 2; ++mt) {
+                  const double af = kk < kx ? X[(8 * mt + lr) * ldx + kk] : 0.0;
+                  dmma(d[mt][0], d[mt][1], af, b);
+                }
+              }
             }
-          }
 #pragma unroll
-          for (int i = 0; i < 2; ++i) {
-            const int col = c0 + 2 * lc + i;
-            if (col < ncol) {
-#pragma unroll
-              for (int mt = 0; mt < 2; ++mt) {
-                const int q1o = 8 * mt + lr;
+            for (int i = 0; i < 2; ++i) {
+              const int col = c0 + 2 * lc + i;
+              if (col < ncol) {
+                double *dst;
+                bool pad = false;
                 if (tab == 2) {
-                  sBr[18 * N * PP + q1o * T + col] = d[mt][i];
+                  dst = sBr + 18 * N * PP + lr * T + col;
                 } else {
-                  const int f = (col % 54) / P, a0 = col % P;
-                  const int fm = 3 * f + (tab == 1 ? 1 : col >= 54 ? 2 : 0);
-                  double *U = sBr + fm * N * PP + q1o * PP + a0;
-                  U[0] = d[mt][i];
-                  if (P < PP && a0 == P - 1) U[1] = 0.0;   // zero pad of the 16-byte pairs
+                  const int fa = (col * 57) >> 9;   // = col / 9 for col < 108
+                  const int a0 = col - fa * P;
+                  const int fm = tab == 1 ? 3 * fa + 1 : (fa < 6 ? 3 * fa : 3 * (fa - 6) + 2);
+                  dst = sBr + fm * N * PP + lr * PP + a0;
+                  pad = P < PP && a0 == P - 1;
+                }
+                const int mstride = tab == 2 ? 8 * T : 8 * PP;   // m-tile 1 = q1 + 8
+#pragma unroll
+                for (int mt = 0; mt < 2; ++mt) {
+                  dst[mt * mstride] = d[mt][i];
+                  if (pad) dst[mt * mstride + 1] = 0.0;   // zero pad of the 16-byte pairs
                 }
               }
             }

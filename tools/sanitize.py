@@ -2,7 +2,7 @@
 """One small corner-force evaluation (or integrator step) for compute-sanitizer.
 
     compute-sanitizer --tool memcheck|racecheck|synccheck python tools/sanitize.py <case>
-cases: c4 (v10.w, 3D k=4, 40 zones), c5 (v11, 3D k=8, 4 zones), c5v8 (v8), c3 (v2.z1m12, 3D k=2),
+cases: c4 (v10.w, 3D k=4, 40 zones), c5 (v11.mb, 3D k=8, 4 zones), c5v8 (v8), c3 (v2.z1m12, 3D k=2),
        c2 (p2d.z2m6, 2D k=4), integrator (2D k=3 RK2 step), host (pipelined host entry, 3D k=2 16^3)."""
 import os
 import sys
@@ -11,7 +11,7 @@ import numpy as np
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
-CASES = {"c4": ("C4", (5, 4, 2), None, "v10.w"), "c5": ("C5", (2, 1, 2), None, "v11"), "c5v8": ("C5", (2, 1, 2), None, "v8"),
+CASES = {"c4": ("C4", (5, 4, 2), None, "v10.w"), "c5": ("C5", (2, 1, 2), None, "v11.mb"), "c5v8": ("C5", (2, 1, 2), None, "v8"),
          "c3": ("C3", (4, 4, 3), None, "v2.z1m12"), "c2": ("C2", (9, 7), None, "p2d.z2m6")}
 
 
@@ -47,6 +47,17 @@ def main(case):
         h.set_rho0detJ0_host(hx[3])
         o = h.eval_host(hx[0], hx[1], hx[2], None)
         print(case, "dt", o[2][0])
+    elif case == "loopback":   # the overlap schedule of the multi-rank exchange (comm streams, events)
+        m, s = synth.config("C3", "S1", N=(8, 6, 6))
+        par = cf.default_params()
+        par.h0 = (1.0 / m.num_zones) ** (1 / 3) / m.order
+        parts = synth.partition(m, 4)
+        hs = [cf.from_synth(m, params=par, part=p, nccl_uid=None) for p in parts]
+        ls = [p.local_state(s) for p in parts]
+        outs = cf.eval_loopback(hs, [t(l.x) for l in ls], [t(l.v) for l in ls], [t(l.e) for l in ls],
+                                [t(l.rho0detJ0) for l in ls])
+        torch.cuda.synchronize()
+        print(case, [h.exchange_schedule() for h in hs], float(outs[0][2].cpu()[0]))
     else:
         raise SystemExit(f"unknown case {case}")
     return 0

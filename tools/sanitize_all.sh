@@ -4,8 +4,8 @@ mkdir -p gpurun_out
 out=gpurun_out/r02_sanitizer.txt
 : > $out
 for tool in memcheck synccheck racecheck; do
-  for c in c4 c5 c5v8 c3 c2 integrator host; do
-    if [ $tool = racecheck ] && [ $c = host ]; then continue; fi
+  for c in c4 c5 c5v8 c3 c2 integrator host loopback; do
+    if [ $tool = racecheck ] && { [ $c = host ] || [ $c = loopback ]; }; then continue; fi
     echo "=== $tool $c" >> $out
     timeout 900 compute-sanitizer --tool $tool --print-limit 20 python tools/sanitize.py $c >> $out 2>&1
     echo "rc=$?" >> $out
