@@ -307,7 +307,46 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
       }
       __syncthreads();
       // ---- stage C^T: q0 -> a0; warps 0-1: d = 0 components (G), 2-4: d != 0 (B), 5: Pq (Phi) -------
-      {
+      if (MB & 4) {
+        // DMMA form (MB bit 2): Y[cd][q1][a0] = sum_q0 X(q0, a0) S[cd][q1][q0] with M = a0 0..7 (one tile),
+        // K = q0 (four steps), N = q1 (two tiles); X = G for d = 0, B otherwise, Phi for the Pq lines (cd = 9,
+        // M = j0).  20 units (cd, q1 tile) over the 8 warps; the a0 = P-1 = 8 row by DFMA on threads 112-255.
+        static_assert(!(MB & 4) || (N == 16 && P == 9 && T == 8), "DMMA stage C^T is written for k = 8");
+        const int lr = lane >> 2, lc = lane & 3;
+#pragma unroll
+        for (int rr = 0; rr < 3; ++rr) {
+          const int u = warp + 8 * rr;
+          if (u < 20) {
+            const int cd = u >> 1, nt = u & 1;
+            const double *X = cd == 9 ? sPhi : (cd % 3 == 0 ? sG : sB);
+            const int ldx = cd == 9 ? Dm::TS : P;
+            const double *Sb = sA + (cd * N + 8 * nt + lr) * SR;   // B[q0][q1 = lr] = S[cd][q1][q0]
+            double d0 = 0.0, d1 = 0.0;
+#pragma unroll
+            for (int ks = 0; ks < 4; ++ks) {
+              const int qq0 = 4 * ks + lc;
+              dmma(d0, d1, X[qq0 * ldx + lr], Sb[qq0]);           // A[a0 = lr][q0 = lc]
+            }
+            const int qa = 8 * nt + 2 * lc;
+            if (cd < 9) {
+              sBr[(cd * N + qa) * P + lr] = d0;
+              sBr[(cd * N + qa + 1) * P + lr] = d1;
+            } else {
+              sBr[9 * N * P + lr * N + qa] = d0;
+              sBr[9 * N * P + lr * N + qa + 1] = d1;
+            }
+          }
+        }
+        if (tid >= NTH - 9 * N) {   // the a0 = 8 row: 144 rows (cd, q1), 16 DFMA each
+          const int it = tid - (NTH - 9 * N), cd = it / N, qq1 = it - cd * N;
+          const double *X = cd % 3 == 0 ? sG : sB;
+          const double *row = sA + (cd * N + qq1) * SR;
+          double y = 0.0;
+#pragma unroll
+          for (int qq0 = 0; qq0 < N; ++qq0) y = fma(X[qq0 * P + P - 1], row[qq0], y);
+          sBr[(cd * N + qq1) * P + P - 1] = y;
+        }
+      } else {
         const CTZ<K> C{3 * o};
         const int grp = warp < 2 ? 0 : warp < 5 ? 1 : warp < 6 ? 2 : 3;
         const int li = (warp - (grp == 0 ? 0 : grp == 1 ? 2 : 5)) * 32 + lane;   // index inside the group
@@ -351,7 +390,61 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
       __syncthreads();
       // ---- stage B^T: q1 -> a1 on all 8 warps: warps 0..NPART-1 ZB items (c, a0) for a1 part = warp,
       //      the next NPART warps ZG items, the rest ZE items (j0) for j1 halves ------------------------
-      {
+      if (MB & 2) {
+        // DMMA form (MB bit 1): ZB[c][a1][a0] = sum_q1 B(q1,a1) Y0[c][q1][a0] + G(q1,a1) Y1[c][q1][a0] and
+        // ZG[c][a1][a0] = sum_q1 B(q1,a1) Y2[c][q1][a0] with M = a1 0..7 (one tile), K = q1 (four steps),
+        // N = (c, a0) columns 9 c + a0 (four tiles, warps 0-3); ZE[j1][j0] = sum_q1 Phi(q1,j1) YE[j0][q1] on
+        // warp 4; the a1 = P-1 = 8 row of ZB / ZG by DFMA on warp 5.
+        static_assert(!(MB & 2) || (N == 16 && P == 9 && T == 8), "DMMA stage B^T is written for k = 8");
+        const int lr = lane >> 2, lc = lane & 3;
+        if (warp < 4) {
+          const int bcol = 8 * warp + lr;                       // this lane's B-operand column (c, a0)
+          const bool bok = bcol < 27;
+          const int bc = (bcol * 57) >> 9, ba0 = bcol - 9 * bc;  // / 9 and % 9 for bcol < 108
+          const double *y0 = sBr + (3 * bc) * N * P + ba0, *y1 = y0 + N * P, *y2 = y0 + 2 * N * P;
+          double zb0 = 0.0, zb1 = 0.0, zg0 = 0.0, zg1 = 0.0;
+#pragma unroll
+          for (int ks = 0; ks < 4; ++ks) {
+            const int qq1 = 4 * ks + lc;
+            const double aB = sB[qq1 * P + lr], aG = sG[qq1 * P + lr];    // A[a1 = lr][q1 = lc]
+            const double b0 = bok ? y0[qq1 * P] : 0.0, b1 = bok ? y1[qq1 * P] : 0.0, b2 = bok ? y2[qq1 * P] : 0.0;
+            dmma(zb0, zb1, aB, b0);
+            dmma(zb0, zb1, aG, b1);
+            dmma(zg0, zg1, aB, b2);
+          }
+#pragma unroll
+          for (int i = 0; i < 2; ++i) {
+            const int col = 8 * warp + 2 * lc + i;
+            if (col < 27) {
+              const int c = (col * 57) >> 9, a0 = col - 9 * c;
+              sA[c * P2 + lr * P + a0] = i ? zb1 : zb0;
+              sA[3 * P2 + c * P2 + lr * P + a0] = i ? zg1 : zg0;
+            }
+          }
+        } else if (warp == 4) {
+          double e0 = 0.0, e1 = 0.0;
+#pragma unroll
+          for (int ks = 0; ks < 4; ++ks) {
+            const int qq1 = 4 * ks + lc;
+            dmma(e0, e1, sPhi[qq1 * Dm::TS + lr], sBr[9 * N * P + lr * N + qq1]);   // A[j1][q1], B[q1][j0 = lr]
+          }
+          sA[6 * P2 + lr * T + 2 * lc] = e0;
+          sA[6 * P2 + lr * T + 2 * lc + 1] = e1;
+        } else if (warp == 5 && lane < 27) {
+          const int c = (lane * 57) >> 9, a0 = lane - 9 * c;
+          const double *y0 = sBr + (3 * c) * N * P + a0, *y1 = y0 + N * P, *y2 = y0 + 2 * N * P;
+          double sb = 0.0, sg = 0.0;
+#pragma unroll
+          for (int qq1 = 0; qq1 < N; ++qq1) {
+            const double bq = sB[qq1 * P + P - 1], gq = sG[qq1 * P + P - 1];
+            sb = fma(bq, y0[qq1 * P], sb);
+            sb = fma(gq, y1[qq1 * P], sb);
+            sg = fma(bq, y2[qq1 * P], sg);
+          }
+          sA[c * P2 + (P - 1) * P + a0] = sb;
+          sA[3 * P2 + c * P2 + (P - 1) * P + a0] = sg;
+        }
+      } else {
         const CTZ<K> C{4 * o};
         if (warp < NPART) {
           if (lane < 3 * P) {
