@@ -91,6 +91,9 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   constexpr bool NOXV = OPT & 32;   // timing diagnostic only (wrong results): no x / v gather
   constexpr bool CLK = !(OPT & 4096);   // per-zone clock64 accounting (BLAST_CF_PROFILE); bit 12 compiles it out
   constexpr int EIG = (OPT & 8192) ? 1 : 0;   // bit 13: branchy smallest eigenpair (pointwise.cuh sym3_min_eig)
+  // bit 14 (RHOPW): rho0|J0| is not staged by the contraction warps (512 of their ~1340 cp.async per zone);
+  // the point warps prefetch zone i+1's into L2 while they work on zone i and load their two values directly
+  constexpr bool RHOPW = OPT & 16384;
   constexpr bool SPREAD = OPT & 64;   // the 6 P^3 node-field copies spread over all contraction threads
   static_assert(!V16 || (Dm::T3 % 2 == 0 && Dm::N3 % 2 == 0 && Dm::XE_E % 2 == 0 && (Dm::OFF_XE + Dm::XE_E) % 2 == 0 &&
                          (Dm::OFF_UV + Dm::O_R) % 2 == 0 && Dm::UVBUF % 2 == 0), "16-byte copies need 16-byte alignment");
@@ -166,7 +169,12 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
         }
       }
       double *R = sUV + (i & 1) * Dm::UVBUF + Dm::O_R;
-      if (BULK) {
+      if (RHOPW) {
+        for (int r = ktid; r < T3 + 10; r += NKW) {
+          const double *src = r < T3 ? a.e + z * T3 + r : r < T3 + 9 ? a.J0inv + z * 9 + (r - T3) : a.zone_gamma + z;
+          cp_async8(sXE + Dm::XE_E + r, src, true);
+        }
+      } else if (BULK) {
         if (ktid == 0) {
           uint64_t *bar = sMB + (i & 1);
           mbar_expect_tx(bar, (T3 + N3) * 8);
@@ -505,7 +513,8 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     const int col = q2 * N + q1;
     const int qa = col * N + q0a, qb = qa + NH;                     // natural point index (R, Sq)
     const int sa = js_idx(col, q0a), sbi = js_idx(col, q0a + NH);  // JS slots
-    const double Ra = ub[Dm::O_R + qa], Rb = ub[Dm::O_R + qb];
+    const double Ra = RHOPW ? __ldg(a.rho0detJ0 + z * N3 + qa) : ub[Dm::O_R + qa];
+    const double Rb = RHOPW ? __ldg(a.rho0detJ0 + z * N3 + qb) : ub[Dm::O_R + qb];
     double ga[9], gb[9];
 #pragma unroll
     for (int i = 0; i < 9; ++i) { ga[i] = 0.0; gb[i] = 0.0; }
@@ -691,6 +700,10 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   long long t_work = 0, t_all = CLK ? clock64() : 0;
   for (int64_t i = 0; i <= nz; ++i) {
     const long long t0 = CLK ? clock64() : 0;
+    if (RHOPW && i + 1 < nz && tid < TPZ) {   // zone i+1's rho0|J0| lines into L2
+      const double *rz = a.rho0detJ0 + zone_of(i + 1) * N3;
+      if ((tid & 7) == 0) asm volatile("prefetch.global.L2 [%0];" ::"l"(rz + 2 * tid));   // 32 lines of 16 doubles
+    }
     if (i < nz && tid < TPZ && DIAG != 2)
       pw_point(sUV + (i & 1) * Dm::UVBUF, sJ + (i & 1) * 10, sJS + (i & 1) * Dm::JSBUF, zone_of(i));
     if (PWG) {   // zone i's points are done: issue zone i+2 (its XE and R slots were last read for zone i)
