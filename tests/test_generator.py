@@ -92,3 +92,25 @@ def test_partition(dim, P):
             other = parts[q]
             assert np.array_equal(np.intersect1d(p.nodes, other.nodes), g)
     assert np.all(owners == 1)   # owner rule: every node counted exactly once
+
+
+@pytest.mark.parametrize("name,N,k,P", [("C4", (8, 6, 4), 2, 8), ("C3", (6, 6, 6), None, 4), ("C2", (10, 8), 3, 8),
+                                        ("C2", (6, 4), 2, 2)])
+def test_partition_numbers_boundary_zones_first(name, N, k, P):
+    """synth.partition numbers each rank's zones boundary-first (the zones touching a node shared with another
+    rank, then the interior ones, each group ascending): the numbering the library's overlap schedule needs
+    (blast_cf_exchange_schedule); every zone appears on exactly one rank."""
+    m, _ = synth.config(name, "S1", N=N, k=k)
+    parts = synth.partition(m, P)
+    seen = np.concatenate([p.zones for p in parts])
+    assert np.array_equal(np.sort(seen), np.arange(m.num_zones))
+    for p in parts:
+        shared = np.zeros(len(p.nodes), dtype=bool)
+        shared[p.nbr_nodes] = True
+        bnd = shared[p.zone_nodes].any(axis=1)
+        nb = int(bnd.sum())
+        assert bnd[:nb].all() and not bnd[nb:].any()
+        assert np.all(np.diff(p.zones[:nb]) > 0) and np.all(np.diff(p.zones[nb:]) > 0)
+        # every rank of a 2 x ... x 2 block partition shares a node with every other (dt piggy-back)
+        if max(synth.block_dims(m.dim, P)) <= 2:
+            assert len(p.nbr_rank) == P - 1
