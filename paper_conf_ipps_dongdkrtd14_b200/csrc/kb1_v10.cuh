@@ -90,7 +90,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4, PWG = OPT & 8, V16 = OPT & 16;
   constexpr bool NOXV = OPT & 32;   // timing diagnostic only (wrong results): no x / v gather
   constexpr bool CLK = !(OPT & 4096);   // per-zone clock64 accounting (BLAST_CF_PROFILE); bit 12 compiles it out
-  constexpr int EIG = (OPT & 8192) ? 1 : 0;   // bit 13: branchy smallest eigenpair (pointwise.cuh sym3_min_eig)
+  constexpr int EIG = (OPT & 8192) ? 1 : (OPT & 32768) ? 2 : 0;   // bits 13 / 15: branchy / warp-uniform shortcut of the eigenpair
   // bit 14 (RHOPW): rho0|J0| is not staged by the contraction warps (512 of their ~1340 cp.async per zone);
   // the point warps prefetch zone i+1's into L2 while they work on zone i and load their two values directly
   constexpr bool RHOPW = OPT & 16384;
