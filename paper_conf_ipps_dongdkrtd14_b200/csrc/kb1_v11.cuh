@@ -313,7 +313,7 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
         // M = j0).  20 units (cd, q1 tile) over the 8 warps; the a0 = P-1 = 8 row by DFMA on threads 112-255.
         static_assert(!(MB & 4) || (N == 16 && P == 9 && T == 8), "DMMA stage C^T is written for k = 8");
         const int lr = lane >> 2, lc = lane & 3;
-#pragma unroll
+#pragma unroll 1
         for (int rr = 0; rr < 3; ++rr) {
           const int u = warp + 8 * rr;
           if (u < 20) {
