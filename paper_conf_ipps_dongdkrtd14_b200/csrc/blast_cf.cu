@@ -483,10 +483,11 @@ int exchange_create(Exchange **out, const blast_cf_mesh *mesh, int dim, int64_t 
 
 int exchange_allreduce_sum2(Exchange *x, double *a, double *b) {
   double hv[2] = {*a, *b};
-  CUDA_TRY(cudaMemcpy(x->d_tmp, hv, sizeof hv, cudaMemcpyHostToDevice));
+  // copies ordered on the NCCL stream (a pageable cudaMemcpy may return before its DMA lands)
+  CUDA_TRY(cudaMemcpyAsync(x->d_tmp, hv, sizeof hv, cudaMemcpyHostToDevice, x->stream));
   NCCL_TRY(x->api->AllReduce(x->d_tmp, x->d_tmp, 2, ncclDouble, ncclSum, x->comm, x->stream), "ncclAllReduce(sum)");
+  CUDA_TRY(cudaMemcpyAsync(hv, x->d_tmp, sizeof hv, cudaMemcpyDeviceToHost, x->stream));
   CUDA_TRY(cudaStreamSynchronize(x->stream));
-  CUDA_TRY(cudaMemcpy(hv, x->d_tmp, sizeof hv, cudaMemcpyDeviceToHost));
   *a = hv[0];
   *b = hv[1];
   return BLAST_CF_OK;
@@ -531,7 +532,7 @@ int exchange_send_rows(Exchange *x, cudaStream_t st, bool with_dt, const double 
 int exchange_run(Exchange *x, double *F1, double *dt) {
   if (!x->comm) return BLAST_CF_OK;   // loopback: blast_cf_eval_loopback moves the data
   exchange_pack(x, F1);
-  const bool all_nbrs = x->num_nbr == x->nranks - 1;   // then the neighbours' dts are every rank's dt
+  const bool all_nbrs = x->dt_piggy;   // every rank neighbours every other (agreed by all ranks at create)
   int rc = exchange_send_rows(x, x->stream, all_nbrs, dt);
   if (rc) return rc;
   if (all_nbrs) {
@@ -820,6 +821,15 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
     if (nccl_unique_id) {
       rc = blastcf::exchange_allreduce_sum2(h->xch, &gvol, &gz);
       if (rc) { free_handle(h); return rc; }
+      // the schedule must be the same on every rank (NCCL calls are matched in order): overlap only if every
+      // rank can, the piggy-backed dt only if every rank neighbours every other
+      double no_overlap = h->xch->overlap ? 0.0 : 1.0, not_all = h->xch->num_nbr == nranks - 1 ? 0.0 : 1.0;
+      rc = blastcf::exchange_allreduce_sum2(h->xch, &no_overlap, &not_all);
+      if (rc) { free_handle(h); return rc; }
+      h->xch->overlap = h->xch->overlap && no_overlap == 0.0;
+      h->xch->dt_piggy = not_all == 0.0;
+    } else {
+      h->xch->dt_piggy = h->xch->num_nbr == nranks - 1;   // loopback: blast_cf_eval_loopback decides per group
     }
   }
   h->h0 = h->params.h0 > 0.0 ? h->params.h0 : pow(gvol / gz, 1.0 / dim) / order;
@@ -866,6 +876,9 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
     if (cudaEventCreate(&e) != cudaSuccess) return bail(fail(BLAST_CF_ECUDA, "event create"));
   if (getenv("BLAST_CF_PROFILE") && cudaMalloc(&h->d_prof, std::max<int64_t>(h->ncta_cap, 1) * 16 * sizeof(long long)) != cudaSuccess)
     return bail(fail(BLAST_CF_ENOMEM, "profile buffer"));
+  // the uploads above are legacy-stream copies from pageable memory: make sure they have landed before any eval
+  // is enqueued on a (possibly non-blocking) user stream
+  if (cudaDeviceSynchronize() != cudaSuccess) return bail(fail(BLAST_CF_ECUDA, "create: %s", cudaGetErrorString(cudaGetLastError())));
   *out = h;
   return BLAST_CF_OK;
 }
@@ -1035,8 +1048,8 @@ static int loopback_move(blast_cf *const *hs, int n) {
       const int64_t cnt = xr->nbr_offset[i + 1] - xr->nbr_offset[i];
       if (iq < 0 || xq->nbr_offset[iq + 1] - xq->nbr_offset[iq] != cnt)
         return fail(BLAST_CF_EINVAL, "ranks %d and %d disagree on their shared nodes", r, q);
-      CUDA_TRY(cudaMemcpy(xr->d_recv + xr->nbr_offset[i] * xr->dim, xq->d_send + xq->nbr_offset[iq] * xq->dim,
-                          cnt * xr->dim * sizeof(double), cudaMemcpyDeviceToDevice));
+      CUDA_TRY(cudaMemcpyAsync(xr->d_recv + xr->nbr_offset[i] * xr->dim, xq->d_send + xq->nbr_offset[iq] * xq->dim,
+                               cnt * xr->dim * sizeof(double), cudaMemcpyDeviceToDevice, hs[r]->stream));
     }
   }
   return BLAST_CF_OK;
@@ -1399,8 +1412,8 @@ int blast_cf_eval_loopback(blast_cf *const *hs, int n, const double *const *x, c
       const int64_t cnt = xr->nbr_offset[i + 1] - xr->nbr_offset[i];
       if (iq < 0 || xq->nbr_offset[iq + 1] - xq->nbr_offset[iq] != cnt)
         return fail(BLAST_CF_EINVAL, "ranks %d and %d disagree on their shared nodes", r, q);
-      CUDA_TRY(cudaMemcpy(xr->d_recv + xr->nbr_offset[i] * xr->dim, xq->d_send + xq->nbr_offset[iq] * xq->dim,
-                          cnt * xr->dim * sizeof(double), cudaMemcpyDeviceToDevice));
+      CUDA_TRY(cudaMemcpyAsync(xr->d_recv + xr->nbr_offset[i] * xr->dim, xq->d_send + xq->nbr_offset[iq] * xq->dim,
+                               cnt * xr->dim * sizeof(double), cudaMemcpyDeviceToDevice, hs[r]->stream));
     }
   }
   // 4. global min dt

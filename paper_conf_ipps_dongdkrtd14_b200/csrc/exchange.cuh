@@ -203,6 +203,7 @@ struct Exchange {
   double *d_rdt = nullptr;       // [num_nbr] neighbours' dt (single-round schedule)
   // overlap schedule: zones [0, nb) touch shared nodes (boundary), [nb, Z) do not (interior)
   bool overlap = false;
+  bool dt_piggy = false;   // single round: every rank neighbours every other, so the dt rides on the F.1 messages
   int64_t nb = 0;
   cudaStream_t s_comm = nullptr;   // high-priority stream of the pack / NCCL / dt work
   cudaEvent_t ev_b = nullptr, ev_i = nullptr, ev_p = nullptr, ev_x = nullptr, ev_sent = nullptr;

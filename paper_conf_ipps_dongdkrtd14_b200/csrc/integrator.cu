@@ -1046,6 +1046,8 @@ int blast_cf_rk2_create(blast_cf *h, const blast_cf_mesh *mesh, const double *rh
   }
 
   // ---- Jacobi diagonal, walls, internal-energy weights ----
+  // the uploads above are legacy-stream copies from pageable memory: let them land before kernels on hv.stream
+  CUDA_TRY(cudaDeviceSynchronize());
   cudaStream_t st = hv.stream;
   if (Z > 0) {
     if (D == 3) {
