@@ -564,7 +564,7 @@ struct blast_cf {
   // host-eval staging (blast_cf_eval_host): device copies of the inputs/outputs and the zone-chunk pipeline
   double *d_in = nullptr, *d_out = nullptr;
   struct HostPipe {
-    static constexpr int MAXC = 8;
+    static constexpr int MAXC = 16;
     const void *plan_for = nullptr;          // KB1 function the plan was built for (autotune may switch it)
     int nch = 0;                             // zone chunks (1 = no pipelining)
     int64_t z0[MAXC + 1] = {};               // chunk c = zones [z0[c], z0[c+1])
@@ -1141,7 +1141,9 @@ static int host_plan(blast_cf *h) {
     resident = std::max(1, occ) * std::max(1, sms);
   }
   const int64_t per_wave = (int64_t)std::max(resident, 1) * std::max(h->var.zpc, 1);
-  int nch = (int)std::min<int64_t>(blast_cf::HostPipe::MAXC, h->Z / (2 * per_wave));
+  const char *env_ch = getenv("BLAST_CF_HOST_CHUNKS");   // default 8 (measured)
+  const int max_ch = std::min(blast_cf::HostPipe::MAXC, env_ch ? std::max(1, atoi(env_ch)) : 8);
+  int nch = (int)std::min<int64_t>(max_ch, h->Z / (2 * per_wave));
   if (h->xch) nch = 1;   // multi-rank: keep the plain path (the exchange follows KB2 anyway)
   nch = std::max(nch, 1);
   std::vector<int32_t> zn((size_t)h->Z * h->nk);
@@ -1248,13 +1250,10 @@ int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const doub
   int64_t gathered = 0;   // nodes [0, gathered) of F.1 are gathered and on their way back
   for (int c = 0; c < P.nch; ++c) {
     const int64_t z0 = P.z0[c], zc = P.z0[c + 1] - z0, n1 = P.hi[c] + 1;
-    if (n1 > done) {
-      for (int d = 0; d < h->dim; ++d) {
-        CUDA_TRY(cudaMemcpyAsync(dx + d * h->nn + done, x + d * h->nn + done, (n1 - done) * sizeof(double),
-                                 cudaMemcpyHostToDevice, P.s_h2d));
-        CUDA_TRY(cudaMemcpyAsync(dv + d * h->nn + done, v + d * h->nn + done, (n1 - done) * sizeof(double),
-                                 cudaMemcpyHostToDevice, P.s_h2d));
-      }
+    if (n1 > done) {   // node range [done, n1) of every component: one 2D copy per array (rows of pitch nn)
+      const size_t pitch = (size_t)h->nn * sizeof(double), w = (size_t)(n1 - done) * sizeof(double);
+      CUDA_TRY(cudaMemcpy2DAsync(dx + done, pitch, x + done, pitch, w, h->dim, cudaMemcpyHostToDevice, P.s_h2d));
+      CUDA_TRY(cudaMemcpy2DAsync(dv + done, pitch, v + done, pitch, w, h->dim, cudaMemcpyHostToDevice, P.s_h2d));
       done = n1;
     }
     CUDA_TRY(cudaMemcpyAsync(de + z0 * h->nt, e + z0 * h->nt, zc * h->nt * sizeof(double), cudaMemcpyHostToDevice, P.s_h2d));
@@ -1280,17 +1279,19 @@ int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const doub
       launch_kb2(h, dF, nullptr, 0, nullptr, h->stream, gathered, g1);
       CUDA_TRY(cudaEventRecord(P.ev_kb1[c], h->stream));
       CUDA_TRY(cudaStreamWaitEvent(P.s_d2h, P.ev_kb1[c], 0));
-      for (int d = 0; d < h->dim; ++d)
-        CUDA_TRY(cudaMemcpyAsync(out_Fdot1 + d * h->nn + gathered, dF + d * h->nn + gathered,
-                                 (g1 - gathered) * sizeof(double), cudaMemcpyDeviceToHost, P.s_d2h));
+      const size_t pitch = (size_t)h->nn * sizeof(double);
+      CUDA_TRY(cudaMemcpy2DAsync(out_Fdot1 + gathered, pitch, dF + gathered, pitch, (g1 - gathered) * sizeof(double), h->dim,
+                                 cudaMemcpyDeviceToHost, P.s_d2h));
       gathered = g1;
     }
   }
   // the remaining nodes and the min dt (nodes above hi[nch-1] belong to no zone: KB2 gives them F.1 = 0)
   launch_kb2(h, dF, P.d_ctadt, P.nslots, dd, h->stream, gathered, h->nn);
-  for (int d = 0; d < h->dim; ++d)
-    CUDA_TRY(cudaMemcpyAsync(out_Fdot1 + d * h->nn + gathered, dF + d * h->nn + gathered, (h->nn - gathered) * sizeof(double),
-                             cudaMemcpyDeviceToHost, h->stream));
+  if (h->nn > gathered) {
+    const size_t pitch = (size_t)h->nn * sizeof(double);
+    CUDA_TRY(cudaMemcpy2DAsync(out_Fdot1 + gathered, pitch, dF + gathered, pitch, (h->nn - gathered) * sizeof(double), h->dim,
+                               cudaMemcpyDeviceToHost, h->stream));
+  }
   CUDA_TRY(cudaMemcpyAsync(out_dt_min, dd, sizeof(double), cudaMemcpyDeviceToHost, h->stream));
   CUDA_TRY(cudaEventRecord(P.ev_d2h, P.s_d2h));
   CUDA_TRY(cudaStreamWaitEvent(h->stream, P.ev_d2h, 0));
