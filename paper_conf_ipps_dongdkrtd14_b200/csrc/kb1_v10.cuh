@@ -94,6 +94,9 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   // bit 14 (RHOPW): rho0|J0| is not staged by the contraction warps (512 of their ~1340 cp.async per zone);
   // the point warps prefetch zone i+1's into L2 while they work on zone i and load their two values directly
   constexpr bool RHOPW = OPT & 16384;
+  // bit 16 (EARLYS): each point's S, P go to the JS buffer right after its evaluation (its J is dead), and the
+  // exact dt of the candidates comes from the J^T J the evaluation kept: point a's S is not live across point b
+  constexpr bool EARLYS = OPT & 65536;
   constexpr bool SPREAD = OPT & 64;   // the 6 P^3 node-field copies spread over all contraction threads
   static_assert(!V16 || (Dm::T3 % 2 == 0 && Dm::N3 % 2 == 0 && Dm::XE_E % 2 == 0 && (Dm::OFF_XE + Dm::XE_E) % 2 == 0 &&
                          (Dm::OFF_UV + Dm::O_R) % 2 == 0 && Dm::UVBUF % 2 == 0), "16-byte copies need 16-byte alignment");
@@ -549,7 +552,20 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     const double w12 = sW[q1] * sW[q2];
     PointOut<3> oa, ob;
     const double best = sRed[8];   // largest exact inverse dt found so far by this CTA (dt filter)
-    if (VMODE == 3 && a.ph.use_visc && a.ph.use_vort) {   // both points one straight-line block, one vote
+    if (EARLYS && VMODE == 3 && a.ph.use_visc && a.ph.use_vort) {
+      point_eval3<2, 1, EIG>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best);
+#pragma unroll
+      for (int cd = 0; cd < 9; ++cd) jb[cd * N3 + sa] = oa.S[cd / 3][cd % 3];
+      jb[Dm::O_PQ + sa] = oa.P;
+      point_eval3<2, 1, EIG>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best);
+#pragma unroll
+      for (int cd = 0; cd < 9; ++cd) jb[cd * N3 + sbi] = ob.S[cd / 3][cd % 3];
+      jb[Dm::O_PQ + sbi] = ob.P;
+      if (__any_sync(0xffffffffu, oa.cand || ob.cand)) {
+        point_dt_exact_m(oa.m, a.ph, oa);
+        point_dt_exact_m(ob.m, a.ph, ob);
+      }
+    } else if (VMODE == 3 && a.ph.use_visc && a.ph.use_vort) {   // both points one straight-line block, one vote
       point_eval3<2, 1, EIG>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best);
       point_eval3<2, 1, EIG>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best);
       if (__any_sync(0xffffffffu, oa.cand || ob.cand)) {   // J is still in the JS buffer (S is written below)
@@ -575,13 +591,15 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       if ((threadIdx.x & 31) == 0 && mi > best)
         atomicMax(reinterpret_cast<unsigned long long *>(sRed + 8), (unsigned long long)__double_as_longlong(mi));
     }
+    if (!(EARLYS && VMODE == 3 && a.ph.use_visc && a.ph.use_vort)) {
 #pragma unroll
-    for (int cd = 0; cd < 9; ++cd) {     // in place over J: only this thread touches slots sa, sbi
-      jb[cd * N3 + sa] = oa.S[cd / 3][cd % 3];
-      jb[cd * N3 + sbi] = ob.S[cd / 3][cd % 3];
+      for (int cd = 0; cd < 9; ++cd) {     // in place over J: only this thread touches slots sa, sbi
+        jb[cd * N3 + sa] = oa.S[cd / 3][cd % 3];
+        jb[cd * N3 + sbi] = ob.S[cd / 3][cd % 3];
+      }
+      jb[Dm::O_PQ + sa] = oa.P;
+      jb[Dm::O_PQ + sbi] = ob.P;
     }
-    jb[Dm::O_PQ + sa] = oa.P;
-    jb[Dm::O_PQ + sbi] = ob.P;
     if (a.Sq != nullptr) {
 #pragma unroll
       for (int cd = 0; cd < 9; ++cd) {
