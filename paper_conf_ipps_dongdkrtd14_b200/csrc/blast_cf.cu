@@ -16,6 +16,7 @@
 #include <vector>
 
 #include "../../include/blast_cf.h"
+#include <nvtx3/nvToolsExt.h>   // header-only NVTX v3: ranges cost nothing unless a tool (nsys, ncu) is attached
 #include "kb1_corner_force.cuh"
 #include "kb1_v2.cuh"
 #include "kb1_v3.cuh"
@@ -34,6 +35,12 @@
 namespace {
 
 thread_local std::string g_last_error;
+
+// NVTX range for the host-side phases (tracing); the kernels themselves are visible to the tools
+struct NvtxRange {
+  explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 int fail(int code, const char *fmt, ...) {
   char buf[512];
@@ -688,6 +695,7 @@ void blast_cf_default_params(blast_cf_params *p) {
 
 int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_cf_params *params,
                     void *cuda_stream, const void *nccl_unique_id, blast_cf **out) {
+  NvtxRange nv("blast_cf_create");
   if (!out) return fail(BLAST_CF_EINVAL, "out is NULL");
   *out = nullptr;
   if (!mesh) return fail(BLAST_CF_EINVAL, "mesh is NULL");
@@ -951,6 +959,7 @@ static void launch_pack_gather(const blast_cf *h, cudaStream_t st) {
 // Overlap schedule of a multi-rank NCCL handle: boundary zones, then the exchange of their
 // shared rows on the comm stream while the interior zones compute; the dt allreduce overlaps KB2.
 static int eval_overlap(blast_cf *h, const KB1Args &a, double *out_Fdot1, double *out_dt_min) {
+  NvtxRange nv("blast_cf_eval: overlap schedule");
   blastcf::Exchange *x = h->xch;
   const int64_t nb = x->nb, ni = h->Z - nb;
   const int gb = range_grid(h, nb, 0), gi = range_grid(h, ni, comm_sms());
@@ -987,6 +996,7 @@ static int eval_impl(blast_cf *h, const double *x, const double *v, const double
   if (rc) return rc;
   const KB1Args a = make_args(h, x, v, e, rho0detJ0, out_FTv, Sq);
   if (h->xch && h->xch->comm && h->xch->overlap) return eval_overlap(h, a, out_Fdot1, out_dt_min);
+  NvtxRange nv("blast_cf_eval");
   if (h->timing) cudaEventRecord(h->ev[0], h->stream);
   if (h->ncta > 0) h->var.launch(a, h->ncta, h->stream);
   if (h->timing) cudaEventRecord(h->ev[1], h->stream);
@@ -1209,6 +1219,7 @@ int blast_cf_set_rho0detJ0_host(blast_cf *h, const double *rho0detJ0) {
 
 int blast_cf_eval_host(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
                        double *out_Fdot1, double *out_FTv, double *out_dt_min) {
+  NvtxRange nv("blast_cf_eval_host");
   if (!h) return fail(BLAST_CF_EINVAL, "handle is NULL");
   if (!out_dt_min || ((!x || !v || !out_Fdot1) && h->nn > 0) || ((!e || !out_FTv) && h->Z > 0))
     return fail(BLAST_CF_EINVAL, "NULL array argument");
