@@ -168,8 +168,10 @@ def test_gpu_invariants():
 # ---------------------------------------------------------------------------------------------
 # BASELINE sizes (the bench's launch configuration): sampled parity
 # ---------------------------------------------------------------------------------------------
-def sampled_parity(orc, name, which, n_nodes=48, n_zones=48, seed=0):
-    m, s = synth.config(name, which)
+def sampled_parity(orc, name, which, n_nodes=48, n_zones=48, seed=0, state=None):
+    m, s = synth.config(name, "S1" if state is not None else which)
+    if state is not None:   # an edge regime of this config's mesh (synth.edge_state)
+        s = synth.edge_state(m, synth.CONFIGS[name]["kind"], state, 7, tie_gap=1.5e-4 if m.order <= 4 else 4.5e-4)
     h, [(F1, FTv, dt)] = gpu_eval(m, s)
     rng = np.random.default_rng(seed)
     nodes = rng.choice(m.num_nodes, size=n_nodes, replace=False)
@@ -210,6 +212,14 @@ def sampled_parity(orc, name, which, n_nodes=48, n_zones=48, seed=0):
                                         ("C5", "S1")])
 def test_full_size_sampled(orc, name, which):
     sampled_parity(orc, name, which, n_nodes=24 if name == "C5" else 48, n_zones=8 if name == "C5" else 48)
+
+
+@pytest.mark.parametrize("name,state", [("C4", "window"), ("C4", "negative_e"), ("C4", "near_tie"),
+                                        ("C5", "negative_e"), ("C3", "near_tie")])
+def test_full_size_sampled_edge_regimes(orc, name, state):
+    """The edge regimes (R25) at the BASELINE sizes, in the bench's launch configuration: sampled nodes and zones
+    against the oracle, the argmin CTA's dt, and the any-size invariants."""
+    sampled_parity(orc, name, None, n_nodes=24 if name == "C5" else 48, n_zones=8 if name == "C5" else 48, state=state)
 
 
 @pytest.mark.parametrize("name", ["v10.v", "v5.r1"])
