@@ -1,11 +1,11 @@
 #!/bin/bash
-# compute-sanitizer memcheck / racecheck / synccheck over the cases of tools/sanitize.py (under gpurun)
+# compute-sanitizer memcheck / racecheck / synccheck / initcheck over the cases of tools/sanitize.py (under gpurun)
 mkdir -p gpurun_out
 out=gpurun_out/r02_sanitizer.txt
 : > $out
-for tool in memcheck synccheck racecheck; do
+for tool in memcheck synccheck racecheck initcheck; do
   for c in c4 c5 c5v8 c3 c2 integrator host loopback; do
-    if [ $tool = racecheck ] && { [ $c = host ] || [ $c = loopback ]; }; then continue; fi
+    if { [ $tool = racecheck ] || [ $tool = initcheck ]; } && { [ $c = host ] || [ $c = loopback ]; }; then continue; fi
     echo "=== $tool $c" >> $out
     timeout 900 compute-sanitizer --tool $tool --print-limit 20 python tools/sanitize.py $c >> $out 2>&1
     echo "rc=$?" >> $out
