@@ -180,9 +180,9 @@ int blast_cf_kernel_times(blast_cf *h, float *ms3);
 /* Multi-rank handles: which exchange schedule eval runs.
  * *mode = 0 (single rank), 1 (single round: KB1, KB2, then one grouped send/recv carrying the F.1 rows
  * and each rank's dt, so no allreduce when every rank neighbours every other) or 2 (overlap: the zones
- * touching shared nodes are numbered first — *boundary_zones of them — and their rows are exchanged on a
- * high-priority comm stream while the interior zones compute on all but BLAST_CF_COMM_SMS (default 4)
- * SMs; the dt allreduce(min) overlaps the node gather).  BLAST_CF_OVERLAP=0 at create forces 1.
+ * touching shared nodes are numbered first — *boundary_zones of them — and run on a high-priority comm
+ * stream concurrently with the interior zones, the resident CTAs split in proportion; their rows are
+ * exchanged while the interior zones compute; the dt allreduce(min) overlaps the node gather).  BLAST_CF_OVERLAP=0 at create forces 1.
  * boundary_zones may be NULL. */
 int blast_cf_exchange_schedule(const blast_cf *h, int32_t *mode, int64_t *boundary_zones);
 /* Tests / profiling, overlap schedule with timing enabled: milliseconds from the start of the last eval to

@@ -463,6 +463,7 @@ int exchange_create(Exchange **out, const blast_cf_mesh *mesh, int dim, int64_t 
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);   // hi = greatest priority (numerically lowest)
     if (cudaStreamCreateWithPriority(&x->s_comm, cudaStreamNonBlocking, hi) != cudaSuccess ||
+        cudaEventCreateWithFlags(&x->ev_s, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&x->ev_b, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&x->ev_i, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&x->ev_p, cudaEventDisableTiming) != cudaSuccess ||
@@ -738,7 +739,7 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
 
   // ---- tables ----
   const blastcf::Tables1D T = blastcf::build_tables(order);
-  const int n = T.n, p = T.p, t = T.t;
+  const int p = T.p;
   std::vector<double> tab;
   tab.insert(tab.end(), T.B.begin(), T.B.end());
   tab.insert(tab.end(), T.G.begin(), T.G.end());
@@ -929,10 +930,23 @@ static int range_grid(const blast_cf *h, int64_t zc, int reserve_sms) {
   return (int)g;
 }
 
-static int comm_sms() {
-  const char *e = getenv("BLAST_CF_COMM_SMS");
-  return e ? std::max(0, atoi(e)) : 4;
+// Overlap schedule: the boundary and the interior zones run CONCURRENTLY as two launches (boundary on the
+// comm stream, interior on the handle's stream); persistent kernels split the resident CTAs in proportion to
+// the zone counts, so both finish together while the boundary rows' exchange runs on the SMs the boundary
+// launch frees (round 2; a boundary-first sequential split paid each launch's pipeline fill twice).
+static void overlap_grids(const blast_cf *h, int64_t nb, int64_t ni, int *gb, int *gi) {
+  if (h->var.persistent && h->ncta >= 2) {
+    const int tot = h->ncta;
+    int b = (int)((double)tot * (double)nb / (double)(nb + ni) + 0.5);
+    b = std::min(std::max(b, 1), tot - 1);
+    *gb = (int)std::min<int64_t>(b, (nb + h->var.zpc - 1) / h->var.zpc);
+    *gi = (int)std::min<int64_t>(tot - b, (ni + h->var.zpc - 1) / h->var.zpc);
+  } else {
+    *gb = range_grid(h, nb, 0);
+    *gi = range_grid(h, ni, 0);
+  }
 }
+
 
 // KB2 on nodes [n0, n1) (default: all); dt != nullptr: its last block also reduces the per-CTA dt slots
 static void launch_kb2(const blast_cf *h, double *F1, const double *cta_dt, int ncta, double *dt, cudaStream_t st,
@@ -962,16 +976,18 @@ static int eval_overlap(blast_cf *h, const KB1Args &a, double *out_Fdot1, double
   NvtxRange nv("blast_cf_eval: overlap schedule");
   blastcf::Exchange *x = h->xch;
   const int64_t nb = x->nb, ni = h->Z - nb;
-  const int gb = range_grid(h, nb, 0), gi = range_grid(h, ni, comm_sms());
+  int gb = 0, gi = 0;
+  overlap_grids(h, nb, ni, &gb, &gi);
   if (h->timing) cudaEventRecord(h->ev[0], h->stream);
-  launch_range(h, a, 0, nb, gb, 0, h->stream);
-  CUDA_TRY(cudaEventRecord(x->ev_b, h->stream));
-  CUDA_TRY(cudaStreamWaitEvent(x->s_comm, x->ev_b, 0));
-  launch_pack_gather(h, x->s_comm);
+  CUDA_TRY(cudaEventRecord(x->ev_s, h->stream));          // the inputs are ready
+  CUDA_TRY(cudaStreamWaitEvent(x->s_comm, x->ev_s, 0));
+  launch_range(h, a, 0, nb, gb, 0, x->s_comm);             // boundary zones (comm stream) ...
+  CUDA_TRY(cudaEventRecord(x->ev_b, x->s_comm));
+  launch_pack_gather(h, x->s_comm);                         // ... then their shared rows out
   int rc = blastcf::exchange_send_rows(x, x->s_comm, false, nullptr);
   if (rc) return rc;
   if (h->timing) cudaEventRecord(x->ev_sent, x->s_comm);
-  launch_range(h, a, nb, ni, gi, gb, h->stream);
+  launch_range(h, a, nb, ni, gi, gb, h->stream);            // interior zones, concurrently (handle's stream)
   CUDA_TRY(cudaEventRecord(x->ev_i, h->stream));
   if (h->timing) cudaEventRecord(h->ev[1], h->stream);
   CUDA_TRY(cudaStreamWaitEvent(x->s_comm, x->ev_i, 0));
@@ -979,6 +995,7 @@ static int eval_overlap(blast_cf *h, const KB1Args &a, double *out_Fdot1, double
   if (x->api->AllReduce(out_dt_min, out_dt_min, 1, ncclDouble, ncclMin, x->comm, x->s_comm) != ncclSuccess)
     return fail(BLAST_CF_ENCCL, "ncclAllReduce(min dt)");
   CUDA_TRY(cudaEventRecord(x->ev_x, x->s_comm));
+  CUDA_TRY(cudaStreamWaitEvent(h->stream, x->ev_b, 0));     // KB2 needs the boundary zones too
   launch_kb2(h, out_Fdot1, nullptr, 0, x->d_tmp, h->stream);   // node gather; dt comes from the comm stream
   if (h->timing) cudaEventRecord(h->ev[2], h->stream);
   CUDA_TRY(cudaStreamWaitEvent(h->stream, x->ev_x, 0));
@@ -1350,12 +1367,12 @@ int blast_cf_eval_loopback(blast_cf *const *hs, int n, const double *const *x, c
       blast_cf *h = hs[r];
       if ((rc = check_async(h))) return rc;
       as[r] = make_args(h, x[r], v[r], e[r], rho0detJ0[r], out_FTv[r], nullptr);
-      gb[r] = range_grid(h, h->xch->nb, 0);
-      gi[r] = range_grid(h, h->Z - h->xch->nb, comm_sms());
+      overlap_grids(h, h->xch->nb, h->Z - h->xch->nb, &gb[r], &gi[r]);
       if (h->timing) cudaEventRecord(h->ev[0], h->stream);
-      launch_range(h, as[r], 0, h->xch->nb, gb[r], 0, h->stream);
-      CUDA_TRY(cudaEventRecord(h->xch->ev_b, h->stream));
-      CUDA_TRY(cudaStreamWaitEvent(h->xch->s_comm, h->xch->ev_b, 0));
+      CUDA_TRY(cudaEventRecord(h->xch->ev_s, h->stream));
+      CUDA_TRY(cudaStreamWaitEvent(h->xch->s_comm, h->xch->ev_s, 0));
+      launch_range(h, as[r], 0, h->xch->nb, gb[r], 0, h->xch->s_comm);   // boundary zones on the comm stream
+      CUDA_TRY(cudaEventRecord(h->xch->ev_b, h->xch->s_comm));
       launch_pack_gather(h, h->xch->s_comm);
       CUDA_TRY(cudaEventRecord(h->xch->ev_p, h->xch->s_comm));
     }
@@ -1385,6 +1402,7 @@ int blast_cf_eval_loopback(blast_cf *const *hs, int n, const double *const *x, c
       CUDA_TRY(cudaStreamWaitEvent(xr->s_comm, xr->ev_i, 0));
       blastcf::xch_dt_reduce<<<1, 256, 0, xr->s_comm>>>(h->d_ctadt, gb[r] + gi[r], out_dt_min[r]);
       CUDA_TRY(cudaEventRecord(xr->ev_x, xr->s_comm));
+      CUDA_TRY(cudaStreamWaitEvent(h->stream, xr->ev_b, 0));
       launch_kb2(h, out_Fdot1[r], nullptr, 0, xr->d_tmp, h->stream);
       if (h->timing) cudaEventRecord(h->ev[2], h->stream);
     }

@@ -206,7 +206,7 @@ struct Exchange {
   bool dt_piggy = false;   // single round: every rank neighbours every other, so the dt rides on the F.1 messages
   int64_t nb = 0;
   cudaStream_t s_comm = nullptr;   // high-priority stream of the pack / NCCL / dt work
-  cudaEvent_t ev_b = nullptr, ev_i = nullptr, ev_p = nullptr, ev_x = nullptr, ev_sent = nullptr;
+  cudaEvent_t ev_s = nullptr, ev_b = nullptr, ev_i = nullptr, ev_p = nullptr, ev_x = nullptr, ev_sent = nullptr;
 };
 
 inline void exchange_destroy(Exchange *x) {
@@ -214,7 +214,7 @@ inline void exchange_destroy(Exchange *x) {
   if (x->comm && x->api) x->api->CommDestroy(x->comm);
   cudaFree(x->d_rows); cudaFree(x->d_unodes); cudaFree(x->d_sptr); cudaFree(x->d_src);
   cudaFree(x->d_send); cudaFree(x->d_recv); cudaFree(x->d_tmp); cudaFree(x->d_rdt);
-  for (cudaEvent_t e : {x->ev_b, x->ev_i, x->ev_p, x->ev_x, x->ev_sent})
+  for (cudaEvent_t e : {x->ev_s, x->ev_b, x->ev_i, x->ev_p, x->ev_x, x->ev_sent})
     if (e) cudaEventDestroy(e);
   if (x->s_comm) cudaStreamDestroy(x->s_comm);
   delete x;
