@@ -750,7 +750,6 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
   std::vector<double> J0inv((size_t)Z * dim * dim);
   long double vol = 0.0L;
   bool affine = true;
-  int64_t bad_zone = -1;
   for (int64_t z = 0; z < Z; ++z) {
     const int32_t *zn = mesh->zone_nodes + z * nk;
     long double J[3][3] = {{0}}, X0[3];
@@ -768,7 +767,7 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
       for (int c = 0; c < dim; ++c) {
         long double xa = X0[c];
         for (int d = 0; d < dim; ++d) xa += J[c][d] * (long double)T.gll[li[d]];
-        if (fabsl(xa - (long double)mesh->x0[c * nn + zn[a]]) > 1e-11L * scale) { affine = false; bad_zone = z; }
+        if (fabsl(xa - (long double)mesh->x0[c * nn + zn[a]]) > 1e-11L * scale) { affine = false; }
       }
     }
     long double det, inv[3][3];
@@ -791,7 +790,6 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
     for (int c = 0; c < dim; ++c)
       for (int d = 0; d < dim; ++d) J0inv[(size_t)z * dim * dim + c * dim + d] = (double)inv[c][d];
   }
-  (void)bad_zone;
   const bool point_j0 = !affine && h->params.use_viscosity;   // reading R19: J0^{-1} at every point
   if (!affine) {   // the mesh volume by quadrature (the vertex-difference det above is exact only for affine zones)
     const int64_t npts = Z * nq;
