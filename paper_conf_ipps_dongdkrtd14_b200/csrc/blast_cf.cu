@@ -1166,8 +1166,8 @@ static int host_plan(blast_cf *h) {
     resident = std::max(1, occ) * std::max(1, sms);
   }
   const int64_t per_wave = (int64_t)std::max(resident, 1) * std::max(h->var.zpc, 1);
-  const char *env_ch = getenv("BLAST_CF_HOST_CHUNKS");   // default 8 (measured)
-  const int max_ch = std::min(blast_cf::HostPipe::MAXC, env_ch ? std::max(1, atoi(env_ch)) : 8);
+  const char *env_ch = getenv("BLAST_CF_HOST_CHUNKS");   // default 6 (measured with the taper below)
+  const int max_ch = std::min(blast_cf::HostPipe::MAXC, env_ch ? std::max(1, atoi(env_ch)) : 6);
   int nch = (int)std::min<int64_t>(max_ch, h->Z / (2 * per_wave));
   if (h->xch) nch = 1;   // multi-rank: keep the plain path (the exchange follows KB2 anyway)
   nch = std::max(nch, 1);
@@ -1177,8 +1177,21 @@ static int host_plan(blast_cf *h) {
   P.nslots = 0;
   int64_t hi = -1;
   for (int c = 0; c < nch; ++c) {
-    P.z0[c] = h->Z * c / nch;
-    P.z0[c + 1] = h->Z * (c + 1) / nch;
+    // chunk sizes taper linearly (weights nch + t - c, t = taper): the last chunk's corner force and copies
+    // are the pipeline's exposed tail, so it is made the smallest
+    const char *tp = getenv("BLAST_CF_HOST_TAPER");
+    const double taper = tp ? atof(tp) : 1.5;
+    auto cum = [&](int cc) {   // sum of the first cc weights / all weights
+      double s_ = 0.0, t_ = 0.0;
+      for (int i = 0; i < nch; ++i) {
+        const double w = taper > 0.0 ? (double)(nch - i) + taper : 1.0;
+        if (i < cc) s_ += w;
+        t_ += w;
+      }
+      return s_ / t_;
+    };
+    P.z0[c] = c == 0 ? 0 : (int64_t)(h->Z * cum(c));
+    P.z0[c + 1] = c + 1 == nch ? h->Z : (int64_t)(h->Z * cum(c + 1));
     for (size_t i = (size_t)P.z0[c] * h->nk; nch > 1 && i < (size_t)P.z0[c + 1] * h->nk; ++i) hi = std::max<int64_t>(hi, zn[i]);
     P.hi[c] = nch > 1 ? hi : h->nn - 1;
     const int64_t zc = P.z0[c + 1] - P.z0[c];
