@@ -1166,8 +1166,8 @@ static int host_plan(blast_cf *h) {
     resident = std::max(1, occ) * std::max(1, sms);
   }
   const int64_t per_wave = (int64_t)std::max(resident, 1) * std::max(h->var.zpc, 1);
-  const char *env_ch = getenv("BLAST_CF_HOST_CHUNKS");   // default 6 (measured with the taper below)
-  const int max_ch = std::min(blast_cf::HostPipe::MAXC, env_ch ? std::max(1, atoi(env_ch)) : 6);
+  const char *env_ch = getenv("BLAST_CF_HOST_CHUNKS");   // default 8 (measured with the taper below)
+  const int max_ch = std::min(blast_cf::HostPipe::MAXC, env_ch ? std::max(1, atoi(env_ch)) : 8);
   int nch = (int)std::min<int64_t>(max_ch, h->Z / (2 * per_wave));
   if (h->xch) nch = 1;   // multi-rank: keep the plain path (the exchange follows KB2 anyway)
   nch = std::max(nch, 1);
