@@ -113,16 +113,6 @@ KB1Variant variant3v3() {
   return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3v3<K, ZPC, MINB>, (const void *)&kb1_v3_3d<K, ZPC, MINB>,
                     false, nullptr};
 }
-template <int K, int MODE>
-void launch3v4(const KB1Args &a, int grid, cudaStream_t s) {
-  using C = KB1V4Cfg<K, MODE>;
-  kb1_v4_3d<K, MODE><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
-}
-template <int K, int MODE>
-KB1Variant variant3v4() {
-  using C = KB1V4Cfg<K, MODE>;
-  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v4<K, MODE>, (const void *)&kb1_v4_3d<K, MODE>, true, nullptr};
-}
 template <int K, int DIAG, int MODE>
 void launch3v5(const KB1Args &a, int grid, cudaStream_t s) {
   using C = KB1V5Cfg<K, MODE>;
@@ -133,16 +123,6 @@ KB1Variant variant3v5() {
   using C = KB1V5Cfg<K, MODE>;
   return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v5<K, DIAG, MODE>, (const void *)&kb1_v5_3d<K, DIAG, MODE>,
                     true, nullptr};
-}
-template <int K, int DIAG>
-void launch3v6(const KB1Args &a, int grid, cudaStream_t s) {
-  using C = KB1V5Cfg<K>;
-  kb1_v6_3d<K, DIAG><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
-}
-template <int K, int DIAG = 0>
-KB1Variant variant3v6() {
-  using C = KB1V5Cfg<K>;
-  return KB1Variant{1, C::NTH, C::SMEM_BYTES, &launch3v6<K, DIAG>, (const void *)&kb1_v6_3d<K, DIAG>, true, nullptr};
 }
 template <int K, int DIAG, int MODE, int OPT, int VMODE>
 void launch3v10(const KB1Args &a, int grid, cudaStream_t s) {
@@ -259,8 +239,6 @@ KB1Variant select_variant(int dim, int k, bool need_point_j0) {
       KB1Variant d;
       if (strcmp(force, "v5.d1") == 0) { d = variant3v5<4, 1>(); d.name = "v5.d1"; return d; }
       if (strcmp(force, "v5.d2") == 0) { d = variant3v5<4, 2>(); d.name = "v5.d2"; return d; }
-      if (strcmp(force, "v6.d1") == 0) { d = variant3v6<4, 1>(); d.name = "v6.d1"; return d; }
-      if (strcmp(force, "v6.d2") == 0) { d = variant3v6<4, 2>(); d.name = "v6.d2"; return d; }
       if (strcmp(force, "v10.q") == 0) { d = variant3v10<4, 0, 0, 4>(); d.name = "v10.q"; return d; }
       if (strcmp(force, "v10.b") == 0) { d = variant3v10<4, 0, 0, 1>(); d.name = "v10.b"; return d; }
       if (strcmp(force, "v10.l") == 0) { d = variant3v10<4, 0, 0, 2>(); d.name = "v10.l"; return d; }
