@@ -386,3 +386,18 @@ def test_point_varying_rho_is_read_per_point(orc):
     s2 = synth.State(s.x, s.v, s.e, np.ascontiguousarray(s.rho0detJ0[:, ::-1]))
     _, [(F1b, FTvb, dtb)] = gpu_eval(m, s2)
     assert rel(F1b, F1) > 1e-6 and rel(FTvb, FTv) > 1e-6
+
+
+def test_non_affine_full_size_host_entry_matches_device():
+    """A curved initial mesh at the C3 size (per-point J0^{-1}, generic kernel) through the pipelined host entry:
+    the zone-chunk shifts of the per-point J0^{-1} array must give the device entry's bits."""
+    torch = _torch()
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    m, s = synth.config("C3", "S1")
+    curved = synth.Mesh(m.dim, m.order, m.N, m.L, s.x.copy(), m.zone_nodes, m.zone_mat, m.mat_gamma)
+    s2 = synth.State(np.ascontiguousarray(s.x + 0.1 * (s.x - m.x0)), s.v, s.e, s.rho0detJ0)
+    h, [(F1, FTv, dt)] = gpu_eval(curved, s2)
+    assert h.variant.startswith("v1")
+    hx = [torch.from_numpy(np.ascontiguousarray(a)).pin_memory() for a in (s2.x, s2.v, s2.e, s2.rho0detJ0)]
+    o = h.eval_host(*hx)
+    assert np.array_equal(o[0], F1) and np.array_equal(o[1], FTv) and o[2][0] == dt
