@@ -245,6 +245,20 @@ def oracle_sample(mesh, st, seconds=15.0, max_zones=None):
     return nz2, t, nthr
 
 
+def kb2_roofline(lmesh, info, kb2_ms):
+    Zl, nn, nk, dim = lmesh.num_zones, lmesh.num_nodes, info["nk"], lmesh.dim
+    bytes_ = 8.0 * Zl * dim * nk + 4.0 * Zl * nk + 4.0 * (nn + 1) + 8.0 * dim * nn
+    peak = None
+    try:
+        peak = float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"])
+        src = "MEASURED_PEAKS.json hbm_gbs"
+    except Exception:
+        peak, src = 6650.0, "B200_PROFILING.md fallback"
+    gbs = bytes_ / (kb2_ms / 1e3) / 1e9 if kb2_ms > 0 else None
+    return {"bound": "hbm", "achieved": gbs, "peak": peak, "unit": "GB/s",
+            "frac": gbs / peak if gbs else None, "bytes": bytes_, "kernel_ms": kb2_ms, "peak_source": src}
+
+
 def run_reference(args):
     rank, world, _ = env_rank()
     if rank != 0:
@@ -477,6 +491,9 @@ def run_ours(args):
                              (f"inputs larger than L2 ({in_bytes / 1e6:.0f} MB of inputs per rank + "
                               f"{Zl * info['nk'] * mesh.dim * 8 / 1e6:.0f} MB zone-local buffer vs {l2_bytes / 1e6:.0f} MB L2); no flush")},
             "gflops": gflops_total,
+            # the node gather (KB2) is HBM-bound: its algorithmic bytes (zone-local F_z.1 + CSR entries + row
+            # pointers read, F.1 written) against the measured copy bandwidth (MEASURED_PEAKS.json hbm_gbs)
+            "kb2_roofline": kb2_roofline(lmesh, info, float(kb[1])),
             "roofline": {"bound": "alu", "achieved": achieved_tf, "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
                          "frac": achieved_tf / FP64_PEAK_TFLOPS, "traffic": traffic,
                          "kernel": f"KB1 (fused corner force, variant {h.variant})",
