@@ -401,3 +401,29 @@ def test_non_affine_full_size_host_entry_matches_device():
     hx = [torch.from_numpy(np.ascontiguousarray(a)).pin_memory() for a in (s2.x, s2.v, s2.e, s2.rho0detJ0)]
     o = h.eval_host(*hx)
     assert np.array_equal(o[0], F1) and np.array_equal(o[1], FTv) and o[2][0] == dt
+
+
+def test_eval_is_cuda_graph_capturable():
+    """include/blast_cf.h: eval is capture-safe for nranks == 1 (bench.py replays small configs from a graph):
+    a captured eval replayed gives the eager eval's bits."""
+    torch = _torch()
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    m, s = synth.config("C2", "S1", N=(32, 32))
+    stream = torch.cuda.Stream()
+    with torch.cuda.stream(stream):
+        h = cf.from_synth(m, stream=stream)
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    x, v, e, r = t(s.x), t(s.v), t(s.e), t(s.rho0detJ0)
+    ref = [o.clone() for o in h.eval(x, v, e, r)]
+    stream.synchronize()
+    out = h.alloc_outputs()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=stream):
+        h.eval(x, v, e, r, out=out)
+    for o in out:
+        o.zero_()
+    with torch.cuda.stream(stream):
+        g.replay()
+    stream.synchronize()
+    for a, b in zip(ref, out):
+        assert torch.equal(a, b)
