@@ -318,6 +318,9 @@ def run_ours(args):
     stream = torch.cuda.Stream(device=dev)
     with torch.cuda.stream(stream):
         h = cf.from_synth(mesh, part=part, nccl_uid=uid, stream=stream) if world > 1 else cf.from_synth(lmesh, stream=stream)
+    if world > 1 and args.transport == "p2p":
+        # the exchange through peer memory (NVLink stores + flags, no NCCL call per eval); NCCL stays for create
+        h.p2p_connect()
     info = h.info
     t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(dev)
     # the states one step evaluates: C2's step is the "full RK2 step RHS" = the corner force at the two
@@ -485,6 +488,9 @@ def run_ours(args):
                        "state": "+".join(["S1", "S1b"][:nev]) if nev > 1 else args.state,
                        "evals_per_step": nev, "zones": Zg, "order": mesh.order, "dim": mesh.dim,
                        "parallelism": f"domain decomposition {synth.block_dims(mesh.dim, world)}" if world > 1 else "single GPU",
+                       "exchange": (f"{h.exchange_transport()} transport, "
+                                    f"{['single rank', 'single round', 'overlap'][h.exchange_schedule()[0]]} schedule")
+                                   if world > 1 else None,
                        "launch": "CUDA-graph replay of the step" if graph is not None else "eager launches",
                        "l2": (f"L2 flushed before every timed step ({work_bytes / 1e6:.0f} MB working set < 2 x "
                               f"{l2_bytes / 1e6:.0f} MB L2; per-step CUDA events)") if flush_l2 else
@@ -534,6 +540,8 @@ def main():
     ap.add_argument("--no-graph", action="store_true", help="launch each step eagerly instead of a CUDA-graph replay")
     ap.add_argument("--no-flush", action="store_true", help="do not flush L2 between timed steps of small configs")
     ap.add_argument("--energy-seconds", type=float, default=2.0)
+    ap.add_argument("--transport", default="p2p", choices=["p2p", "nccl"],
+                    help="N > 1: the shared-DOF exchange through peer memory (default) or NCCL send/recv + allreduce")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

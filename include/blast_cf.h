@@ -185,6 +185,35 @@ int blast_cf_kernel_times(blast_cf *h, float *ms3);
  * exchanged while the interior zones compute; the dt allreduce(min) overlaps the node gather).  BLAST_CF_OVERLAP=0 at create forces 1.
  * boundary_zones may be NULL. */
 int blast_cf_exchange_schedule(const blast_cf *h, int32_t *mode, int64_t *boundary_zones);
+
+/* Peer-memory transport of the exchange (SURVEY §8(e) phase 2; the MFEM shared-DOF assembly and MPI
+ * min-dt of PAPER.md:772-798, the limiter named at PAPER.md:873-876).  Instead of packing the shared rows
+ * for ncclSend / ncclRecv and reducing dt with ncclAllReduce, the kernel that computes a shared row stores
+ * it straight into the neighbour's receive mailbox (CUDA IPC mapping: NVLink / NVSwitch loads and stores)
+ * and releases a system-scope flag; each rank's dt is written into every other rank's mailbox the same
+ * way; the combine kernel acquires the flags and sums in ascending rank order, so the results are bitwise
+ * those of the NCCL transport.  No NCCL call is made per eval; both schedules of blast_cf_exchange_schedule
+ * apply (the schedule is re-agreed at connect: overlap only if every rank can).
+ * Bootstrap (collective over the caller's process group, e.g. torch.distributed with any backend):
+ *   1. every rank: blast_cf_p2p_export(h, NULL, &bytes) for the record size, then
+ *      blast_cf_p2p_export(h, record, &bytes) — allocates and zero-fills this rank's mailbox and describes
+ *      it (IPC handle, process id, device, shared-row offsets) in `record` (host memory, `bytes` long);
+ *   2. all-gather the records in rank order (rank r of the group = mesh->rank r);
+ *   3. every rank: blast_cf_p2p_connect(h, records, bytes) — maps the other ranks' mailboxes
+ *      (cudaIpcOpenMemHandle; plain pointers for handles of the same process) and checks that both sides
+ *      of every neighbour pair agree on the shared-row counts.
+ * The handle must have nranks > 1 (created with an NCCL id, or as a loopback handle: no NCCL needed at
+ * all then, params->h0 must be given).  Afterwards every rank must call blast_cf_eval equally often (an
+ * eval waits for its neighbours' rows of the same eval; a neighbour that never sends makes the eval's
+ * kernel trap after ~30 s instead of hanging), and before blast_cf_destroy the ranks must synchronize
+ * (stream sync + a process-group barrier): a peer may still be writing into this rank's mailbox until
+ * its own eval has finished.  eval with a connected handle is not CUDA-graph capturable (the eval number
+ * is a kernel argument).  Errors: EINVAL (bad / inconsistent records, connect twice, single-rank handle),
+ * EUNSUPPORTED (no peer access between the devices), ECUDA (IPC mapping failed). */
+int blast_cf_p2p_export(blast_cf *h, void *record, int64_t *bytes);
+int blast_cf_p2p_connect(blast_cf *h, const void *records, int64_t bytes_each);
+/* *transport = 0 (single rank), 1 (NCCL), 2 (loopback group, tests), 3 (peer memory, blast_cf_p2p_connect) */
+int blast_cf_exchange_transport(const blast_cf *h, int32_t *transport);
 /* Tests / profiling, overlap schedule with timing enabled: milliseconds from the start of the last eval to
  * [0] the end of the shared-row exchange (comm stream), [1] the end of the interior zones' corner force,
  * [2] the end of the eval.  [0] < [1] shows the exchange hidden behind the interior compute. */

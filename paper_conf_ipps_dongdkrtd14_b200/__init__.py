@@ -104,6 +104,9 @@ def lib():
     L.blast_cf_debug_cta_dt.argtypes = [vp, vp, i64, ctypes.POINTER(i32), ctypes.POINTER(i32)]
     L.blast_cf_debug_stage_clocks.argtypes = [vp, vp, i64]
     L.blast_cf_eval_loopback.argtypes = [vp, ctypes.c_int, vp, vp, vp, vp, vp, vp, vp]
+    L.blast_cf_p2p_export.argtypes = [vp, vp, ctypes.POINTER(i64)]
+    L.blast_cf_p2p_connect.argtypes = [vp, vp, i64]
+    L.blast_cf_exchange_transport.argtypes = [vp, ctypes.POINTER(i32)]
     L.blast_cf_autotune.argtypes = [vp] * 8 + [ctypes.c_int, vp, ctypes.c_int, ctypes.POINTER(ctypes.c_int)]
     L.blast_cf_variant_name.argtypes = [vp, ctypes.c_int]
     L.blast_cf_variant_name.restype = ctypes.c_char_p
@@ -129,7 +132,8 @@ def lib():
               "blast_cf_exchange_schedule", "blast_cf_debug_exchange_times", "blast_cf_eval_debug_Fz", "blast_cf_get_info",
               "blast_cf_set_timing", "blast_cf_kernel_times", "blast_cf_destroy", "blast_cf_nccl_unique_id_size",
               "blast_cf_nccl_get_unique_id", "blast_cf_exchange_plan", "blast_cf_owner_mask", "blast_cf_debug_cta_dt",
-              "blast_cf_debug_stage_clocks", "blast_cf_eval_loopback", "blast_cf_autotune"):
+              "blast_cf_debug_stage_clocks", "blast_cf_eval_loopback", "blast_cf_autotune", "blast_cf_p2p_export",
+              "blast_cf_p2p_connect", "blast_cf_exchange_transport"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
     return L
@@ -361,6 +365,31 @@ class CornerForce:
         _check(lib().blast_cf_exchange_schedule(self._h, ctypes.byref(mode), ctypes.byref(nb)), "blast_cf_exchange_schedule")
         return mode.value, nb.value
 
+    TRANSPORTS = {0: "single rank", 1: "nccl", 2: "loopback", 3: "p2p"}
+
+    def exchange_transport(self) -> str:
+        """How eval moves the shared rows and dt: blast_cf_exchange_transport."""
+        t = ctypes.c_int32(0)
+        _check(lib().blast_cf_exchange_transport(self._h, ctypes.byref(t)), "blast_cf_exchange_transport")
+        return self.TRANSPORTS[t.value]
+
+    def p2p_connect(self, group=None):
+        """Switch the exchange to the peer-memory transport (blast_cf_p2p_export / _connect): a collective over
+        the torch process group `group` (any backend; its rank r must be mesh rank r).  The records are
+        all-gathered as opaque bytes; the library maps the peers' mailboxes itself."""
+        import torch.distributed as dist
+        L = lib()
+        n = ctypes.c_int64(0)
+        _check(L.blast_cf_p2p_export(self._h, None, ctypes.byref(n)), "blast_cf_p2p_export")
+        buf = ctypes.create_string_buffer(n.value)
+        _check(L.blast_cf_p2p_export(self._h, buf, ctypes.byref(n)), "blast_cf_p2p_export")
+        recs = [None] * dist.get_world_size(group)
+        dist.all_gather_object(recs, buf.raw, group=group)
+        allr = b"".join(recs)
+        _check(L.blast_cf_p2p_connect(self._h, allr, n.value), "blast_cf_p2p_connect")
+        self._p2p_group = group if group is not None else dist.group.WORLD
+        self.info = self.get_info()   # kernels_per_eval of the new transport
+
     def debug_exchange_times(self):
         ms = (ctypes.c_float * 3)()
         _check(lib().blast_cf_debug_exchange_times(self._h, ms), "blast_cf_debug_exchange_times")
@@ -375,13 +404,28 @@ class CornerForce:
         return list(ms)
 
     def close(self):
+        """Destroy the handle.  A peer-memory connected handle first synchronizes its device and waits for the
+        whole process group (a peer may still be writing into this rank's mailbox), so every rank must call
+        close() explicitly; without that (garbage collection) its mailbox is left allocated."""
         if getattr(self, "_h", None):
+            if getattr(self, "_p2p_group", None) is not None:
+                import torch
+                import torch.distributed as dist
+                torch.cuda.synchronize(self.device)
+                dist.barrier(group=self._p2p_group)
+                self._p2p_group = None
             lib().blast_cf_destroy(self._h)
             self._h = None
 
+    def _abandon(self):   # garbage collection of a connected handle: never free a mailbox a peer may write
+        self._h = None
+
     def __del__(self):
         try:
-            self.close()
+            if getattr(self, "_p2p_group", None) is not None:
+                self._abandon()
+            else:
+                self.close()
         except Exception:
             pass
 

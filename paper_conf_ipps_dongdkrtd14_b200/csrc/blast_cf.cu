@@ -6,6 +6,8 @@
 // stream, plus the shared-DOF exchange when nranks > 1 (exchange.cuh).  No allocation in eval.
 #include <cuda_runtime.h>
 
+#include <unistd.h>
+
 #include <algorithm>
 #include <cmath>
 #include <cstdarg>
@@ -980,6 +982,58 @@ static int eval_overlap(blast_cf *h, const KB1Args &a, double *out_Fdot1, double
   return check_async(h);
 }
 
+// Peer-memory transport (p2p.cuh): the shared rows are computed by the kernel that stores
+// them into the neighbours' mailboxes, the dt goes to every rank's mailbox, the combine acquires both.
+// Overlap schedule as eval_overlap (boundary zones on the comm stream beside the interior zones; the rows
+// leave as soon as the boundary zones are done); otherwise one round after KB1 and KB2.  No NCCL call.
+static int eval_p2p(blast_cf *h, const KB1Args &a, double *out_Fdot1, double *out_dt_min) {
+  NvtxRange nv("blast_cf_eval: peer-memory exchange");
+  blastcf::Exchange *x = h->xch;
+  blastcf::P2PHost &p = x->p2p;
+  const uint64_t E = ++p.epoch;
+  auto send_rows = [&](cudaStream_t st) {
+    if (x->num_nbr > 0)
+      blastcf::p2p_send_rows<<<p.send_blocks, 256, 0, st>>>(h->d_Fz1, h->d_ptr, h->d_ent, h->nk, h->dim, x->d_rows, p.dev, E);
+  };
+  auto combine = [&](cudaStream_t st) {
+    blastcf::p2p_combine<<<p.combine_blocks, 256, 0, st>>>(out_Fdot1, h->nn, h->dim, x->d_unodes, x->nu, x->d_sptr,
+                                                          x->d_src, out_dt_min, p.dev, E);
+  };
+  if (h->timing) cudaEventRecord(h->ev[0], h->stream);
+  if (x->overlap) {
+    const int64_t nb = x->nb, ni = h->Z - nb;
+    int gb = 0, gi = 0;
+    overlap_grids(h, nb, ni, &gb, &gi);
+    CUDA_TRY(cudaEventRecord(x->ev_s, h->stream));
+    CUDA_TRY(cudaStreamWaitEvent(x->s_comm, x->ev_s, 0));
+    launch_range(h, a, 0, nb, gb, 0, x->s_comm);             // boundary zones (comm stream) ...
+    CUDA_TRY(cudaEventRecord(x->ev_b, x->s_comm));
+    send_rows(x->s_comm);                                     // ... their rows straight into the neighbours
+    if (h->timing) cudaEventRecord(x->ev_sent, x->s_comm);
+    launch_range(h, a, nb, ni, gi, gb, h->stream);            // interior zones, concurrently
+    CUDA_TRY(cudaEventRecord(x->ev_i, h->stream));
+    if (h->timing) cudaEventRecord(h->ev[1], h->stream);
+    CUDA_TRY(cudaStreamWaitEvent(x->s_comm, x->ev_i, 0));
+    blastcf::p2p_send_dt<<<1, 256, 0, x->s_comm>>>(h->d_ctadt, gb + gi, out_dt_min, p.dev, E);
+    CUDA_TRY(cudaEventRecord(x->ev_x, x->s_comm));
+    CUDA_TRY(cudaStreamWaitEvent(h->stream, x->ev_b, 0));
+    launch_kb2(h, out_Fdot1, nullptr, 0, nullptr, h->stream);
+    if (h->timing) cudaEventRecord(h->ev[2], h->stream);
+    CUDA_TRY(cudaStreamWaitEvent(h->stream, x->ev_x, 0));
+    combine(h->stream);
+  } else {
+    if (h->ncta > 0) h->var.launch(a, h->ncta, h->stream);
+    if (h->timing) cudaEventRecord(h->ev[1], h->stream);
+    launch_kb2(h, out_Fdot1, nullptr, 0, nullptr, h->stream);
+    if (h->timing) cudaEventRecord(h->ev[2], h->stream);
+    send_rows(h->stream);
+    blastcf::p2p_send_dt<<<1, 256, 0, h->stream>>>(h->d_ctadt, h->ncta, out_dt_min, p.dev, E);
+    combine(h->stream);
+  }
+  if (h->timing) cudaEventRecord(h->ev[3], h->stream);
+  return check_async(h);
+}
+
 static int eval_impl(blast_cf *h, const double *x, const double *v, const double *e, const double *rho0detJ0,
                      double *out_Fdot1, double *out_FTv, double *out_dt_min, double *Sq) {
   if (!h) return fail(BLAST_CF_EINVAL, "handle is NULL");
@@ -988,6 +1042,7 @@ static int eval_impl(blast_cf *h, const double *x, const double *v, const double
   int rc = check_async(h);
   if (rc) return rc;
   const KB1Args a = make_args(h, x, v, e, rho0detJ0, out_FTv, Sq);
+  if (h->xch && h->xch->p2p.connected) return eval_p2p(h, a, out_Fdot1, out_dt_min);
   if (h->xch && h->xch->comm && h->xch->overlap) return eval_overlap(h, a, out_Fdot1, out_dt_min);
   NvtxRange nv("blast_cf_eval");
   if (h->timing) cudaEventRecord(h->ev[0], h->stream);
@@ -1032,7 +1087,8 @@ static int check_group(blast_cf *const *hs, int n, bool *loop) {
   *loop = hs[0]->xch && !hs[0]->xch->comm;
   if (!*loop) return n == 1 ? BLAST_CF_OK : fail(BLAST_CF_EINVAL, "an NCCL group call drives one rank (n = 1)");
   for (int r = 0; r < n; ++r)
-    if (!hs[r] || !hs[r]->xch || hs[r]->xch->comm || hs[r]->xch->nranks != n || hs[r]->xch->rank != r)
+    if (!hs[r] || !hs[r]->xch || hs[r]->xch->comm || hs[r]->xch->p2p.connected || hs[r]->xch->nranks != n ||
+        hs[r]->xch->rank != r)
       return fail(BLAST_CF_EINVAL, "handle %d is not rank %d of a %d-rank loopback group", r, r, n);
   return BLAST_CF_OK;
 }
@@ -1525,6 +1581,212 @@ int blast_cf_exchange_schedule(const blast_cf *h, int32_t *mode, int64_t *bounda
   if (!h || !mode) return fail(BLAST_CF_EINVAL, "NULL argument");
   *mode = h->xch ? (h->xch->overlap ? 2 : 1) : 0;
   if (boundary_zones) *boundary_zones = h->xch ? h->xch->nb : 0;
+  return BLAST_CF_OK;
+}
+
+// ---- peer-memory transport (p2p.cuh) ----
+namespace {
+struct P2PRecord {   // + int64 recv_off[nranks], recv_cnt[nranks]
+  char magic[8];
+  cudaIpcMemHandle_t mem;
+  uint64_t dptr;
+  int32_t pid, device, rank, nranks, dim, overlap;
+  int64_t nrows, mbox_bytes;
+};
+size_t p2p_record_bytes(int nranks) { return sizeof(P2PRecord) + 2 * sizeof(int64_t) * (size_t)nranks; }
+struct DeviceGuard {   // the calling thread's current device, restored on return
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) == cudaSuccess && prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+struct MboxLayout {   // byte offsets inside a mailbox (p2p.cuh)
+  size_t rows, dt, flag_rows, flag_dt, ack, total;
+};
+MboxLayout mbox_layout(int64_t nrows, int dim, int nranks) {
+  MboxLayout L;
+  L.rows = 0;
+  L.dt = L.rows + 2 * (size_t)std::max<int64_t>(nrows, 0) * dim * sizeof(double);
+  L.flag_rows = L.dt + 2 * (size_t)nranks * sizeof(double);
+  L.flag_dt = L.flag_rows + (size_t)nranks * sizeof(uint64_t);
+  L.ack = L.flag_dt + (size_t)nranks * sizeof(uint64_t);
+  L.total = L.ack + (size_t)nranks * sizeof(uint64_t);
+  return L;
+}
+}  // namespace
+
+int blast_cf_p2p_export(blast_cf *h, void *record, int64_t *bytes) {
+  if (!h || !bytes) return fail(BLAST_CF_EINVAL, "NULL argument");
+  if (!h->xch) return fail(BLAST_CF_EINVAL, "single-rank handle: nothing to exchange");
+  blastcf::Exchange *x = h->xch;
+  const size_t need = p2p_record_bytes(x->nranks);
+  if (!record) {
+    *bytes = (int64_t)need;
+    return BLAST_CF_OK;
+  }
+  if (*bytes < (int64_t)need) return fail(BLAST_CF_EINVAL, "record buffer of %lld bytes, need %zu", (long long)*bytes, need);
+  if (x->p2p.connected) return fail(BLAST_CF_EINVAL, "already connected");
+  DeviceGuard dg(h->device);
+  const MboxLayout L = mbox_layout(x->nrows, x->dim, x->nranks);
+  if (!x->p2p.mbox) {
+    CUDA_TRY(cudaMalloc(&x->p2p.mbox, L.total));
+    x->p2p.mbox_bytes = L.total;
+  }
+  // zero flags / acks before any peer can see the mailbox (its record leaves this process only after this)
+  CUDA_TRY(cudaMemsetAsync(x->p2p.mbox, 0, L.total, h->stream));
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  std::vector<char> buf(need, 0);
+  P2PRecord *r = reinterpret_cast<P2PRecord *>(buf.data());
+  memcpy(r->magic, "BLASTP2P", 8);
+  CUDA_TRY(cudaIpcGetMemHandle(&r->mem, x->p2p.mbox));
+  r->dptr = (uint64_t)(uintptr_t)x->p2p.mbox;
+  r->pid = (int32_t)getpid(); r->device = h->device; r->rank = x->rank; r->nranks = x->nranks; r->dim = x->dim;
+  r->overlap = x->overlap ? 1 : 0; r->nrows = x->nrows; r->mbox_bytes = (int64_t)L.total;
+  int64_t *off = reinterpret_cast<int64_t *>(r + 1), *cnt = off + x->nranks;
+  for (int t = 0; t < x->nranks; ++t) { off[t] = -1; cnt[t] = 0; }
+  for (int i = 0; i < x->num_nbr; ++i) {
+    off[x->nbr_rank[i]] = x->nbr_offset[i];
+    cnt[x->nbr_rank[i]] = x->nbr_offset[i + 1] - x->nbr_offset[i];
+  }
+  memcpy(record, buf.data(), need);
+  *bytes = (int64_t)need;
+  return BLAST_CF_OK;
+}
+
+int blast_cf_p2p_connect(blast_cf *h, const void *records, int64_t bytes_each) {
+  if (!h || !records) return fail(BLAST_CF_EINVAL, "NULL argument");
+  if (!h->xch) return fail(BLAST_CF_EINVAL, "single-rank handle: nothing to exchange");
+  blastcf::Exchange *x = h->xch;
+  blastcf::P2PHost &p = x->p2p;
+  const int n = x->nranks, me = x->rank;
+  if (bytes_each != (int64_t)p2p_record_bytes(n)) return fail(BLAST_CF_EINVAL, "record size %lld", (long long)bytes_each);
+  if (!p.mbox || p.connected) return fail(BLAST_CF_EINVAL, "export first, connect once");
+  auto rec = [&](int t) { return reinterpret_cast<const P2PRecord *>(static_cast<const char *>(records) + (size_t)t * bytes_each); };
+  auto roff = [&](int t) { return reinterpret_cast<const int64_t *>(rec(t) + 1); };
+  for (int t = 0; t < n; ++t) {
+    const P2PRecord *r = rec(t);
+    if (memcmp(r->magic, "BLASTP2P", 8) != 0 || r->rank != t || r->nranks != n || r->dim != x->dim)
+      return fail(BLAST_CF_EINVAL, "record %d is not rank %d of this %d-rank group", t, t, n);
+  }
+  if (rec(me)->dptr != (uint64_t)(uintptr_t)p.mbox || rec(me)->pid != (int32_t)getpid())
+    return fail(BLAST_CF_EINVAL, "record %d is not this handle's", me);
+  for (int i = 0; i < x->num_nbr; ++i) {   // both sides must agree on every shared row count
+    const int q = x->nbr_rank[i];
+    const int64_t mine = x->nbr_offset[i + 1] - x->nbr_offset[i];
+    if (roff(q)[n + me] != mine || roff(q)[me] < 0)
+      return fail(BLAST_CF_EINVAL, "ranks %d and %d disagree on their shared nodes", me, q);
+  }
+  DeviceGuard dg(h->device);
+  p.peer.assign(n, nullptr);
+  p.ipc_opened.assign(n, 0);
+  for (int t = 0; t < n; ++t) {
+    if (t == me) continue;
+    const P2PRecord *r = rec(t);
+    if (r->pid == (int32_t)getpid()) {   // same process: the allocation is addressable as is
+      if (r->device != h->device) {
+        int ok = 0;
+        CUDA_TRY(cudaDeviceCanAccessPeer(&ok, h->device, r->device));
+        if (!ok) return fail(BLAST_CF_EUNSUPPORTED, "device %d cannot access device %d", h->device, r->device);
+        const cudaError_t e = cudaDeviceEnablePeerAccess(r->device, 0);
+        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) CUDA_TRY(e);
+        cudaGetLastError();
+      }
+      p.peer[t] = (void *)(uintptr_t)r->dptr;
+    } else {   // another process (device ordinals need not match across processes: the IPC open checks access)
+      const cudaError_t e = cudaIpcOpenMemHandle(&p.peer[t], r->mem, cudaIpcMemLazyEnablePeerAccess);
+      if (e != cudaSuccess) {
+        p.peer[t] = nullptr;
+        return fail(BLAST_CF_ECUDA, "cudaIpcOpenMemHandle(rank %d): %s", t, cudaGetErrorString(e));
+      }
+      p.ipc_opened[t] = 1;
+    }
+  }
+  // device tables
+  std::vector<double *> row_dst(std::max(x->num_nbr, 1), nullptr), dt_dst(n, nullptr);
+  std::vector<int64_t> row_ps(std::max(x->num_nbr, 1), 0);
+  std::vector<uint64_t *> row_flag(std::max(x->num_nbr, 1), nullptr), dt_flag(n, nullptr), ack_dst(n, nullptr);
+  std::vector<int32_t> blk_off(x->num_nbr + 1, 0);
+  for (int i = 0; i < x->num_nbr; ++i) {
+    const int q = x->nbr_rank[i];
+    const P2PRecord *r = rec(q);
+    const MboxLayout Lq = mbox_layout(r->nrows, x->dim, n);
+    row_dst[i] = reinterpret_cast<double *>(static_cast<char *>(p.peer[q]) + Lq.rows) + roff(q)[me] * x->dim;
+    row_ps[i] = r->nrows * x->dim;
+    row_flag[i] = reinterpret_cast<uint64_t *>(static_cast<char *>(p.peer[q]) + Lq.flag_rows) + me;
+    const int64_t cnt = x->nbr_offset[i + 1] - x->nbr_offset[i];
+    blk_off[i + 1] = blk_off[i] + (int32_t)std::min<int64_t>(std::max<int64_t>((cnt + 255) / 256, 1), 64);
+  }
+  for (int t = 0; t < n; ++t) {
+    if (t == me) continue;
+    const MboxLayout Lt = mbox_layout(rec(t)->nrows, x->dim, n);
+    char *b = static_cast<char *>(p.peer[t]);
+    dt_dst[t] = reinterpret_cast<double *>(b + Lt.dt);
+    dt_flag[t] = reinterpret_cast<uint64_t *>(b + Lt.flag_dt) + me;
+    ack_dst[t] = reinterpret_cast<uint64_t *>(b + Lt.ack) + me;
+  }
+  const size_t nn1 = std::max(x->num_nbr, 1);
+  const size_t sz = nn1 * (sizeof(double *) + sizeof(int64_t) + sizeof(uint64_t *) + sizeof(int64_t) + sizeof(int32_t)) +
+                    (size_t)n * (sizeof(double *) + 2 * sizeof(uint64_t *)) + (nn1 + 1) * sizeof(int32_t) +
+                    (nn1 + 1) * sizeof(int32_t) + 64;
+  CUDA_TRY(cudaMalloc(&p.d_tab, sz));
+  CUDA_TRY(cudaMemset(p.d_tab, 0, sz));
+  char *d = static_cast<char *>(p.d_tab);
+  size_t o = 0;
+  auto put = [&](const void *src, size_t bytes) -> void * {
+    o = (o + 7) / 8 * 8;
+    void *dst = d + o;
+    if (bytes) cudaMemcpy(dst, src, bytes, cudaMemcpyHostToDevice);
+    o += bytes;
+    return dst;
+  };
+  std::vector<int64_t> nbr_off(x->nbr_offset.begin(), x->nbr_offset.end());
+  if (nbr_off.empty()) nbr_off.push_back(0);
+  std::vector<int32_t> nbr_rank(x->nbr_rank.begin(), x->nbr_rank.end());
+  if (nbr_rank.empty()) nbr_rank.push_back(-1);
+  blastcf::P2PDev &g = p.dev;
+  g.row_dst = static_cast<double *const *>(put(row_dst.data(), nn1 * sizeof(double *)));
+  g.row_pstride = static_cast<const int64_t *>(put(row_ps.data(), nn1 * sizeof(int64_t)));
+  g.row_flag = static_cast<uint64_t *const *>(put(row_flag.data(), nn1 * sizeof(uint64_t *)));
+  g.nbr_off = static_cast<const int64_t *>(put(nbr_off.data(), nbr_off.size() * sizeof(int64_t)));
+  g.nbr_rank = static_cast<const int32_t *>(put(nbr_rank.data(), nbr_rank.size() * sizeof(int32_t)));
+  g.blk_off = static_cast<const int32_t *>(put(blk_off.data(), blk_off.size() * sizeof(int32_t)));
+  std::vector<int32_t> zeros(nn1 + 1, 0);
+  g.cnt = static_cast<int32_t *>(put(zeros.data(), nn1 * sizeof(int32_t)));
+  g.done = static_cast<int32_t *>(put(zeros.data(), sizeof(int32_t)));
+  g.dt_dst = static_cast<double *const *>(put(dt_dst.data(), n * sizeof(double *)));
+  g.dt_flag = static_cast<uint64_t *const *>(put(dt_flag.data(), n * sizeof(uint64_t *)));
+  g.ack_dst = static_cast<uint64_t *const *>(put(ack_dst.data(), n * sizeof(uint64_t *)));
+  if (o > sz) return fail(BLAST_CF_ECUDA, "p2p table overflow");
+  CUDA_TRY(cudaGetLastError());
+  g.num_nbr = x->num_nbr;
+  const MboxLayout L = mbox_layout(x->nrows, x->dim, n);
+  char *mb = static_cast<char *>(p.mbox);
+  g.rows = reinterpret_cast<const double *>(mb + L.rows);
+  g.rows_pstride = x->nrows * x->dim;
+  g.dt = reinterpret_cast<const double *>(mb + L.dt);
+  g.flag_rows = reinterpret_cast<const uint64_t *>(mb + L.flag_rows);
+  g.flag_dt = reinterpret_cast<const uint64_t *>(mb + L.flag_dt);
+  g.ack = reinterpret_cast<const uint64_t *>(mb + L.ack);
+  g.me = me;
+  g.nranks = n;
+  p.send_blocks = blk_off[x->num_nbr];
+  p.combine_blocks = (int)std::min<int64_t>(std::max<int64_t>((x->nu + 255) / 256, 1), 1184);
+  // the schedule: overlap only if every rank can (the records carry each rank's own decision)
+  bool all_overlap = true;
+  for (int t = 0; t < n; ++t) all_overlap = all_overlap && rec(t)->overlap;
+  x->overlap = all_overlap && x->overlap;
+  p.epoch = 0;
+  p.connected = true;
+  CUDA_TRY(cudaDeviceSynchronize());
+  return BLAST_CF_OK;
+}
+
+int blast_cf_exchange_transport(const blast_cf *h, int32_t *transport) {
+  if (!h || !transport) return fail(BLAST_CF_EINVAL, "NULL argument");
+  *transport = !h->xch ? 0 : h->xch->p2p.connected ? 3 : h->xch->comm ? 1 : 2;
   return BLAST_CF_OK;
 }
 

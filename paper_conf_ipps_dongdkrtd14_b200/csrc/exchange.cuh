@@ -25,6 +25,7 @@
 #include <vector>
 
 #include "nccl.h"
+#include "p2p.cuh"
 
 namespace blastcf {
 
@@ -138,10 +139,14 @@ __global__ void xch_combine(double *__restrict__ F1, int64_t nn, int dim, const 
     for (int64_t i = sptr[u]; i < sptr[u + 1]; ++i) {
       const int64_t code = src[i];
       const double *row = code >= 0 ? send + code * dim : recv + (-code - 1) * dim;
-      for (int c = 0; c < dim; ++c) s[c] += row[c];
+#pragma unroll
+      for (int c = 0; c < 3; ++c)   // (c < 3 unrolled: s stays in registers)
+        if (c < dim) s[c] += row[c];
     }
     const int64_t node = unodes[u];
-    for (int c = 0; c < dim; ++c) F1[c * nn + node] = s[c];
+#pragma unroll
+    for (int c = 0; c < 3; ++c)
+      if (c < dim) F1[c * nn + node] = s[c];
   }
 }
 
@@ -156,9 +161,13 @@ __global__ void xch_pack_gather(const double *__restrict__ Fz1, const int32_t *_
     double s[3] = {0.0, 0.0, 0.0};
     for (int i = ptr[node]; i < ptr[node + 1]; ++i) {
       const int o = ent[i];
-      for (int c = 0; c < dim; ++c) s[c] += Fz1[o + c * nk];
+#pragma unroll
+      for (int c = 0; c < 3; ++c)
+        if (c < dim) s[c] += Fz1[o + c * nk];
     }
-    for (int c = 0; c < dim; ++c) send[r * dim + c] = s[c];
+#pragma unroll
+    for (int c = 0; c < 3; ++c)
+      if (c < dim) send[r * dim + c] = s[c];
   }
 }
 
@@ -188,6 +197,19 @@ __global__ void xch_dt_combine(double *__restrict__ dt, const double *__restrict
   }
 }
 
+// peer-memory transport (p2p.cuh), set up by blast_cf_p2p_connect
+struct P2PHost {
+  void *mbox = nullptr;           // this rank's mailbox
+  size_t mbox_bytes = 0;
+  std::vector<void *> peer;       // mapped mailboxes of the other ranks (nullptr for this rank)
+  std::vector<char> ipc_opened;   // 1: cudaIpcOpenMemHandle'd (closed at destroy)
+  void *d_tab = nullptr;          // device tables of P2PDev (pointers, strides, counters)
+  P2PDev dev{};
+  uint64_t epoch = 0;             // evals run so far (the next one is epoch + 1)
+  int send_blocks = 0, combine_blocks = 1;
+  bool connected = false;
+};
+
 struct Exchange {
   NcclApi *api = nullptr;
   ncclComm_t comm = nullptr;
@@ -207,10 +229,14 @@ struct Exchange {
   int64_t nb = 0;
   cudaStream_t s_comm = nullptr;   // high-priority stream of the pack / NCCL / dt work
   cudaEvent_t ev_s = nullptr, ev_b = nullptr, ev_i = nullptr, ev_p = nullptr, ev_x = nullptr, ev_sent = nullptr;
+  P2PHost p2p;   // p2p.connected: eval moves the rows and dt through peer memory, no NCCL call
 };
 
 inline void exchange_destroy(Exchange *x) {
   if (!x) return;
+  for (size_t t = 0; t < x->p2p.peer.size(); ++t)
+    if (x->p2p.ipc_opened[t]) cudaIpcCloseMemHandle(x->p2p.peer[t]);
+  cudaFree(x->p2p.mbox); cudaFree(x->p2p.d_tab);
   if (x->comm && x->api) x->api->CommDestroy(x->comm);
   cudaFree(x->d_rows); cudaFree(x->d_unodes); cudaFree(x->d_sptr); cudaFree(x->d_src);
   cudaFree(x->d_send); cudaFree(x->d_recv); cudaFree(x->d_tmp); cudaFree(x->d_rdt);
@@ -222,6 +248,8 @@ inline void exchange_destroy(Exchange *x) {
 
 // kernels of ours one eval launches besides KB1 / KB2 (NCCL's own kernels not counted)
 inline int exchange_kernels(const Exchange *x) {
+  if (x->p2p.connected)   // send rows (num_nbr > 0) + send dt + combine, plus the second KB1 launch of the overlap schedule
+    return (x->overlap ? 1 : 0) + (x->num_nbr > 0 ? 1 : 0) + 2;
   const int combine = x->nu > 0 ? 1 : 0, pack = x->nrows > 0 ? 1 : 0;
   return x->overlap ? 1 /* second KB1 launch */ + pack + 1 /* dt reduce */ + combine : pack + combine + 1 /* dt combine */;
 }

@@ -140,7 +140,7 @@ def test_loopback_schedules_bitwise_equal_and_overlap_visible(monkeypatch):
             assert np.array_equal(x, y)
 
 
-def _nccl_worker(rank, world, uid, overlap, q):
+def _nccl_worker(rank, world, uid, overlap, q, transport="nccl", port=0):
     import os
     os.environ["BLAST_CF_OVERLAP"] = overlap
     import torch
@@ -149,6 +149,12 @@ def _nccl_worker(rank, world, uid, overlap, q):
     m, s = synth.config("C3", "S1", N=(8, 6, 6))
     part = synth.partition(m, world)[rank]
     h = cf.from_synth(m, part=part, nccl_uid=uid)
+    if transport == "p2p":   # NCCL for create, peer memory for every eval (bootstrap all-gather over gloo)
+        import torch.distributed as dist
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        h.p2p_connect()
+        assert h.exchange_transport() == "p2p"
     ls = part.local_state(s)
     t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
     outs = None
@@ -159,11 +165,13 @@ def _nccl_worker(rank, world, uid, overlap, q):
     h.close()
 
 
+@pytest.mark.parametrize("transport", ["nccl", "p2p"])
 @pytest.mark.parametrize("overlap", ["1", "0"])
-def test_nccl_multiprocess(orc, overlap):
-    """The real NCCL path: P = min(#GPUs, 8) processes, one per GPU, both schedules; every rank's F.1 matches
-    the single-domain oracle, sharers hold the same bits, dt is the global min.  Needs >= 2 GPUs (NCCL
-    refuses two ranks on one device)."""
+def test_nccl_multiprocess(orc, overlap, transport):
+    """The real NCCL path: P = min(#GPUs, 8) processes, one per GPU, both schedules, the exchange by NCCL or
+    through peer memory (NCCL then only at create); every rank's F.1 matches the single-domain oracle,
+    sharers hold the same bits, dt is the global min.  Needs >= 2 GPUs (NCCL refuses two ranks on one
+    device; the peer-memory transport alone is tested on one GPU in test_gpu_p2p.py)."""
     import torch
     if not torch.cuda.is_available() or torch.cuda.device_count() < 2:
         pytest.skip("needs >= 2 GPUs")
@@ -173,7 +181,11 @@ def test_nccl_multiprocess(orc, overlap):
     uid = cf.nccl_unique_id()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_nccl_worker, args=(r, P, uid, overlap, q)) for r in range(P)]
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    procs = [ctx.Process(target=_nccl_worker, args=(r, P, uid, overlap, q, transport, port)) for r in range(P)]
     for p in procs:
         p.start()
     got = sorted(q.get(timeout=300) for _ in range(P))
