@@ -320,7 +320,7 @@ def run_ours(args):
         h = cf.from_synth(mesh, part=part, nccl_uid=uid, stream=stream) if world > 1 else cf.from_synth(lmesh, stream=stream)
     if world > 1 and args.transport == "p2p":
         # the exchange through peer memory (NVLink stores + flags, no NCCL call per eval); NCCL stays for create
-        h.p2p_connect()
+        h.p2p_connect(required=False)   # every rank stays on NCCL if the mapping failed anywhere
     info = h.info
     t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(dev)
     # the states one step evaluates: C2's step is the "full RK2 step RHS" = the corner force at the two

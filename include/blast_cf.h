@@ -212,6 +212,10 @@ int blast_cf_exchange_schedule(const blast_cf *h, int32_t *mode, int64_t *bounda
  * EUNSUPPORTED (no peer access between the devices), ECUDA (IPC mapping failed). */
 int blast_cf_p2p_export(blast_cf *h, void *record, int64_t *bytes);
 int blast_cf_p2p_connect(blast_cf *h, const void *records, int64_t bytes_each);
+/* Switch a connected handle back to NCCL (enable = 0; needs the NCCL communicator of create) or to peer
+ * memory again (1).  Every rank must make the same choice before its next eval — e.g. when the connect
+ * failed on some rank, all ranks fall back.  Synchronizes the handle's stream.  EINVAL otherwise. */
+int blast_cf_p2p_enable(blast_cf *h, int enable);
 /* *transport = 0 (single rank), 1 (NCCL), 2 (loopback group, tests), 3 (peer memory, blast_cf_p2p_connect) */
 int blast_cf_exchange_transport(const blast_cf *h, int32_t *transport);
 /* Tests / profiling, overlap schedule with timing enabled: milliseconds from the start of the last eval to

@@ -107,6 +107,7 @@ def lib():
     L.blast_cf_p2p_export.argtypes = [vp, vp, ctypes.POINTER(i64)]
     L.blast_cf_p2p_connect.argtypes = [vp, vp, i64]
     L.blast_cf_exchange_transport.argtypes = [vp, ctypes.POINTER(i32)]
+    L.blast_cf_p2p_enable.argtypes = [vp, ctypes.c_int]
     L.blast_cf_autotune.argtypes = [vp] * 8 + [ctypes.c_int, vp, ctypes.c_int, ctypes.POINTER(ctypes.c_int)]
     L.blast_cf_variant_name.argtypes = [vp, ctypes.c_int]
     L.blast_cf_variant_name.restype = ctypes.c_char_p
@@ -133,7 +134,7 @@ def lib():
               "blast_cf_set_timing", "blast_cf_kernel_times", "blast_cf_destroy", "blast_cf_nccl_unique_id_size",
               "blast_cf_nccl_get_unique_id", "blast_cf_exchange_plan", "blast_cf_owner_mask", "blast_cf_debug_cta_dt",
               "blast_cf_debug_stage_clocks", "blast_cf_eval_loopback", "blast_cf_autotune", "blast_cf_p2p_export",
-              "blast_cf_p2p_connect", "blast_cf_exchange_transport"):
+              "blast_cf_p2p_connect", "blast_cf_exchange_transport", "blast_cf_p2p_enable"):
         getattr(L, f).restype = ctypes.c_int
     _lib = L
     return L
@@ -373,10 +374,12 @@ class CornerForce:
         _check(lib().blast_cf_exchange_transport(self._h, ctypes.byref(t)), "blast_cf_exchange_transport")
         return self.TRANSPORTS[t.value]
 
-    def p2p_connect(self, group=None):
+    def p2p_connect(self, group=None, required=True):
         """Switch the exchange to the peer-memory transport (blast_cf_p2p_export / _connect): a collective over
         the torch process group `group` (any backend; its rank r must be mesh rank r).  The records are
-        all-gathered as opaque bytes; the library maps the peers' mailboxes itself."""
+        all-gathered as opaque bytes; the library maps the peers' mailboxes itself.  All ranks agree on the
+        outcome: if the mapping failed on any rank, every rank stays on NCCL (needs the NCCL communicator of
+        create) and, with required=True, raises.  Returns whether the peer-memory transport is in use."""
         import torch.distributed as dist
         L = lib()
         n = ctypes.c_int64(0)
@@ -385,10 +388,21 @@ class CornerForce:
         _check(L.blast_cf_p2p_export(self._h, buf, ctypes.byref(n)), "blast_cf_p2p_export")
         recs = [None] * dist.get_world_size(group)
         dist.all_gather_object(recs, buf.raw, group=group)
-        allr = b"".join(recs)
-        _check(L.blast_cf_p2p_connect(self._h, allr, n.value), "blast_cf_p2p_connect")
-        self._p2p_group = group if group is not None else dist.group.WORLD
+        rc = L.blast_cf_p2p_connect(self._h, b"".join(recs), n.value)
+        err = None if rc == 0 else f"blast_cf_p2p_connect: {L.blast_cf_last_error().decode()}"
+        errs = [None] * len(recs)
+        dist.all_gather_object(errs, err, group=group)
+        failed = [e for e in errs if e is not None]
+        self._p2p_group = group if group is not None else dist.group.WORLD   # the mailbox exists either way
+        if failed:
+            if rc == 0:
+                _check(L.blast_cf_p2p_enable(self._h, 0), "blast_cf_p2p_enable")
+            if required:
+                raise RuntimeError(f"peer-memory transport unavailable: {failed[0]}")
+            self.p2p_error = failed[0]
+            return False
         self.info = self.get_info()   # kernels_per_eval of the new transport
+        return True
 
     def debug_exchange_times(self):
         ms = (ctypes.c_float * 3)()

@@ -1628,7 +1628,7 @@ int blast_cf_p2p_export(blast_cf *h, void *record, int64_t *bytes) {
     return BLAST_CF_OK;
   }
   if (*bytes < (int64_t)need) return fail(BLAST_CF_EINVAL, "record buffer of %lld bytes, need %zu", (long long)*bytes, need);
-  if (x->p2p.connected) return fail(BLAST_CF_EINVAL, "already connected");
+  if (x->p2p.mapped) return fail(BLAST_CF_EINVAL, "already connected");
   DeviceGuard dg(h->device);
   const MboxLayout L = mbox_layout(x->nrows, x->dim, x->nranks);
   if (!x->p2p.mbox) {
@@ -1663,7 +1663,7 @@ int blast_cf_p2p_connect(blast_cf *h, const void *records, int64_t bytes_each) {
   blastcf::P2PHost &p = x->p2p;
   const int n = x->nranks, me = x->rank;
   if (bytes_each != (int64_t)p2p_record_bytes(n)) return fail(BLAST_CF_EINVAL, "record size %lld", (long long)bytes_each);
-  if (!p.mbox || p.connected) return fail(BLAST_CF_EINVAL, "export first, connect once");
+  if (!p.mbox || p.mapped || !p.peer.empty()) return fail(BLAST_CF_EINVAL, "export first, connect once");
   auto rec = [&](int t) { return reinterpret_cast<const P2PRecord *>(static_cast<const char *>(records) + (size_t)t * bytes_each); };
   auto roff = [&](int t) { return reinterpret_cast<const int64_t *>(rec(t) + 1); };
   for (int t = 0; t < n; ++t) {
@@ -1779,8 +1779,19 @@ int blast_cf_p2p_connect(blast_cf *h, const void *records, int64_t bytes_each) {
   for (int t = 0; t < n; ++t) all_overlap = all_overlap && rec(t)->overlap;
   x->overlap = all_overlap && x->overlap;
   p.epoch = 0;
+  p.mapped = true;
   p.connected = true;
   CUDA_TRY(cudaDeviceSynchronize());
+  return BLAST_CF_OK;
+}
+
+int blast_cf_p2p_enable(blast_cf *h, int enable) {
+  if (!h || !h->xch) return fail(BLAST_CF_EINVAL, "not a multi-rank handle");
+  blastcf::P2PHost &p = h->xch->p2p;
+  if (enable && !p.mapped) return fail(BLAST_CF_EINVAL, "not connected");
+  if (!enable && !h->xch->comm) return fail(BLAST_CF_EINVAL, "no NCCL communicator to fall back to");
+  CUDA_TRY(cudaStreamSynchronize(h->stream));
+  p.connected = enable != 0;
   return BLAST_CF_OK;
 }
 

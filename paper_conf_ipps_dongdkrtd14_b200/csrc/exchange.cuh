@@ -207,7 +207,8 @@ struct P2PHost {
   P2PDev dev{};
   uint64_t epoch = 0;             // evals run so far (the next one is epoch + 1)
   int send_blocks = 0, combine_blocks = 1;
-  bool connected = false;
+  bool mapped = false;      // connect succeeded
+  bool connected = false;   // eval uses this transport (blast_cf_p2p_enable can switch back to NCCL)
 };
 
 struct Exchange {

@@ -92,3 +92,36 @@ def test_p2p_multiprocess(tmp_path, name, N, k, P, overlap):
                     assert np.array_equal(shared[key], val), (r, it, g)   # every sharer holds the same bits
                 else:
                     shared[key] = val
+
+
+def test_p2p_connect_errors():
+    """blast_cf_p2p_*: the error paths (include/blast_cf.h) — single-rank handle, enable before connect,
+    a record of the wrong size or not from this group, a fall-back without an NCCL communicator."""
+    import ctypes
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ipps_dongdkrtd14_b200 as cf
+    import synth
+    L = cf.lib()
+    m, _ = synth.config("C3", "S1", N=(4, 4, 4))
+    h1 = cf.from_synth(m)
+    n = ctypes.c_int64(0)
+    assert L.blast_cf_p2p_export(h1._h, None, ctypes.byref(n)) == 1          # single rank: EINVAL
+    par = cf.default_params()
+    par.h0 = h1.info["h0"]
+    parts = synth.partition(m, 2)
+    h = cf.from_synth(m, params=par, part=parts[0], nccl_uid=None)
+    assert L.blast_cf_p2p_enable(h._h, 1) == 1                              # not connected
+    assert L.blast_cf_p2p_export(h._h, None, ctypes.byref(n)) == 0 and n.value > 0
+    small = ctypes.c_int64(n.value - 1)
+    buf = ctypes.create_string_buffer(n.value)
+    assert L.blast_cf_p2p_export(h._h, buf, ctypes.byref(small)) == 1        # buffer too small
+    assert L.blast_cf_p2p_export(h._h, buf, ctypes.byref(n)) == 0
+    assert L.blast_cf_p2p_connect(h._h, buf.raw * 2, n.value - 8) == 1       # wrong record size
+    assert L.blast_cf_p2p_connect(h._h, buf.raw * 2, n.value) == 1           # record 1 is not rank 1's
+    assert L.blast_cf_p2p_connect(h._h, b"\0" * (2 * n.value), n.value) == 1  # not records at all
+    assert L.blast_cf_p2p_enable(h._h, 0) == 1                              # no NCCL communicator
+    assert h.exchange_transport() == "loopback"
+    h.close()
+    h1.close()
