@@ -47,6 +47,12 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
   static_assert(P % 3 == 0 || P == 8, "stage B^T: a1 split in three parts of P/3 (k = 8) or two of 4 (k = 7)");
   static_assert(3 * P <= 32, "stage B^T: one (c, a0) item per lane");
   constexpr int NPART = P % 3 == 0 ? 3 : 2, PL = P / NPART;   // B^T: a1 parts per item
+  // MB bit 4 (SDT): the CTA's min dt is kept in shared memory (one warp-min + atomicMin per warp and slab)
+  // instead of a register pair + flag live across the whole zone loop.  At the 128-register cap those were
+  // spilled and reloaded in stages A and C, whose loads then missed the small L1 (2 CTAs x ~100 KB of shared
+  // memory per SM): ncu put 7 % of v11.mbt's stall samples on those reloads (long scoreboard).  48 -> 24 B
+  // of spills (what is left sits inside the eigen-solve), 13.73 -> 12.88 ms on C5.
+  constexpr bool SDT = MB & 16;
   extern __shared__ double smem[];
   double *sB = smem, *sG = sB + N * P, *sPhi = sG + N * P, *sW = sPhi + N * Dm::TS;
   double *sF = smem + Dm::OFF_FIX;
@@ -83,6 +89,7 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
   for (int r = tid; r < 3 * NK; r += NTH) sAF[r] = 0.0;
   for (int r = tid; r < NT; r += NTH) sAE[r] = 0.0;
   if (tid == 0) sRed[8] = 0.0;   // dt filter: the CTA's best exact inverse dt
+  if (SDT && tid == 0) sRed[10] = __longlong_as_double(0x7ff0000000000000LL);   // SDT: the CTA's min dt
   if (nz > 0) gather(0);
   cp_async_commit();
   cp_async_wait<0>();
@@ -253,6 +260,7 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
       }
       __syncthreads();
       // ---- stage C (a0 -> q0) + point evaluation ----------------------------------------------------
+      double dslab = __longlong_as_double(0x7ff0000000000000LL);   // SDT: this thread's dt of the slab (0: det J <= 0)
       if (has_point) {
         double g18[18];
 #pragma unroll
@@ -302,8 +310,18 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
 #pragma unroll
           for (int cd = 0; cd < 9; ++cd) a.Sq[(z * (int64_t)(N * NS) + q) * 9 + cd] = pt.S[cd / 3][cd % 3];
         }
-        dtmin = fmin(dtmin, pt.dt);
-        bad |= pt.bad;
+        if (SDT) {
+          dslab = pt.bad ? 0.0 : pt.dt;
+        } else {
+          dtmin = fmin(dtmin, pt.dt);
+          bad |= pt.bad;
+        }
+      }
+      if (SDT) {   // dt >= 0: doubles order like their bit patterns, so an integer min is the min
+#pragma unroll
+        for (int sft = 16; sft > 0; sft >>= 1) dslab = fmin(dslab, __shfl_xor_sync(0xffffffffu, dslab, sft));
+        if (lane == 0)
+          atomicMin(reinterpret_cast<unsigned long long *>(sRed + 10), (unsigned long long)__double_as_longlong(dslab));
       }
       __syncthreads();
       // ---- stage C^T: q0 -> a0; warps 0-1: d = 0 components (G), 2-4: d != 0 (B), 5: Pq (Phi) -------
@@ -525,6 +543,10 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
     for (int i = tid; i < NT; i += NTH) { a.FTv[z * NT + i] = sAE[i]; sAE[i] = 0.0; }
     cp_async_wait<0>();   // the next zone's X, V, e, J0^{-1} (issued in the last slab)
     __syncthreads();
+  }
+  if (SDT) {   // the last __syncthreads of the zone loop ordered every warp's atomicMin before this read
+    if (tid == 0) a.cta_dt[blockIdx.x] = nz > 0 ? sRed[10] : __longlong_as_double(0x7ff0000000000000LL);
+    return;
   }
   if (bad) dtmin = 0.0;
   const double m = block_min(dtmin, sRed);
