@@ -202,7 +202,7 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
       case 6: add(variant3<6, 1, 2>(), "v1.z1m2"); add(variant3<6, 2, 1>(), "v1.z2"); break;
       case 7: add(variant3v8<7, 1>(), "v8"); add(variant3v11<7, 1>(), "v11"); add(variant3<7, 1, 2>(), "v1.z1"); break;
-      case 8: add(variant3v11<8, 2, 19>(), "v11.mbts"); add(variant3v11<8, 2, 3>(), "v11.mbt"); add(variant3v11<8, 2, 1>(), "v11.mb"); add(variant3v8<8, 2>(), "v8"); add(variant3v11<8, 2>(), "v11"); add(variant3v8<8, 1>(), "v8.m1"); add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
+      case 8: add(variant3v11<8, 2, 83>(), "v11.mbtsi"); add(variant3v11<8, 2, 19>(), "v11.mbts"); add(variant3v11<8, 2, 3>(), "v11.mbt"); add(variant3v11<8, 2, 1>(), "v11.mb"); add(variant3v8<8, 2>(), "v8"); add(variant3v11<8, 2>(), "v11"); add(variant3v8<8, 1>(), "v8.m1"); add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
     }
   } else {
     switch (k) {

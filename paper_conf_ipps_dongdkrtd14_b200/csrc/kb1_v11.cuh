@@ -61,7 +61,10 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
 
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int64_t Z = a.num_zones, nn = a.num_nodes, G = gridDim.x;
-  const int64_t nz = Z > blockIdx.x ? (Z - 1 - blockIdx.x) / G + 1 : 0;
+  // MB bit 6 (I32): the zone loop counter in 32 bits (fewer registers live across the point stage; zone
+  // offsets are still formed in 64 bits)
+  using ZI = typename std::conditional<(MB & 64) != 0, int, int64_t>::type;
+  const ZI nz = (ZI)(Z > blockIdx.x ? (Z - 1 - blockIdx.x) / G + 1 : 0);
   auto zone_of = [&](int64_t i) { return (int64_t)blockIdx.x + i * G; };
 
   // gather of zone i (cp.async; the caller commits / waits): X, V [6][NK], e [NT], J0^{-1} + gamma
@@ -101,7 +104,7 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
   bool bad = false;
 
 #pragma unroll 1
-  for (int64_t zi = 0; zi < nz; ++zi) {
+  for (ZI zi = 0; zi < nz; ++zi) {
     const int64_t z = zone_of(zi);
     const double *sJ0 = sJ0b + (zi & 1) * 10;
     const bool more = zi + 1 < nz;
