@@ -41,7 +41,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     objs, procs = [], []
     for src in SOURCES:   # one object per translation unit, compiled in parallel
         obj = os.path.join(OBJDIR, os.path.basename(src) + f".{os.getpid()}.o")
-        cmd = ["nvcc", *NVCC_FLAGS, *inc, "-c", "-o", obj, src]
+        # BLAST_CF_NVCC_FLAGS: extra flags for experiments (e.g. -DBLAST_CF_DIAGNOSTICS, timing-only kernels)
+        cmd = ["nvcc", *NVCC_FLAGS, *os.environ.get("BLAST_CF_NVCC_FLAGS", "").split(), *inc, "-c", "-o", obj, src]
         if verbose:
             cmd.insert(1, "-Xptxas=-v")
             print(" ".join(cmd))

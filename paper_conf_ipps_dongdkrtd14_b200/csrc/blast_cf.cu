@@ -196,6 +196,8 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
         // (round 2: the superseded generations v10 (runtime switches), v10.wu, v6, v5, v4.m0/m1, v3.z1 that never
         //  won the autotuner are no longer instantiated; DESIGN.md §10 keeps their measurements)
         add(variant3v10<4, 0, 0, 0, 3>(), "v10.w");
+        add(variant3v10<4, 0, 0, (1 << 25), 3>(), "v10.wp");
+        add(variant3v10<4, 0, 0, (1 << 26), 3>(), "v10.wph");
         add(variant3v10<4, 0, 0, 0, 2>(), "v10.v"); add(variant3v5<4, 0, 1>(), "v5.r1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;
@@ -261,6 +263,25 @@ KB1Variant select_variant(int dim, int k, bool need_point_j0) {
       if (strcmp(force, "v10.wd1") == 0) { d = variant3v10<4, 1, 0, 0, 3>(); d.name = "v10.wd1"; return d; }
       if (strcmp(force, "v10.vd1") == 0) { d = variant3v10<4, 1, 0, 0, 2>(); d.name = "v10.vd1"; return d; }
       if (strcmp(force, "v10.d1") == 0) { d = variant3v10<4, 1>(); d.name = "v10.d1"; return d; }
+      if (strcmp(force, "v10.wdt0") == 0) { d = variant3v10<4, 0, 0, 131072, 3>(); d.name = "v10.wdt0"; return d; }
+      if (strcmp(force, "v10.wdt1") == 0) { d = variant3v10<4, 0, 0, 262144, 3>(); d.name = "v10.wdt1"; return d; }
+      if (strcmp(force, "v10.wnc") == 0) { d = variant3v10<4, 0, 0, 524288, 3>(); d.name = "v10.wnc"; return d; }
+      if (strcmp(force, "v10.wd2") == 0) { d = variant3v10<4, 2, 0, 0, 3>(); d.name = "v10.wd2"; return d; }
+      if (strcmp(force, "v10.wd3") == 0) { d = variant3v10<4, 3, 0, 0, 3>(); d.name = "v10.wd3"; return d; }
+      if (strcmp(force, "v10.wd3nc") == 0) { d = variant3v10<4, 3, 0, 524288, 3>(); d.name = "v10.wd3nc"; return d; }
+      if (strcmp(force, "v10.wd3ne") == 0) { d = variant3v10<4, 3, 0, 2097152, 3>(); d.name = "v10.wd3ne"; return d; }
+      if (strcmp(force, "v10.wd3ncv") == 0) { d = variant3v10<4, 3, 0, 1048576, 3>(); d.name = "v10.wd3ncv"; return d; }
+      if (strcmp(force, "v10.wd3x") == 0) { d = variant3v10<4, 3, 0, 1048576 | 2097152, 3>(); d.name = "v10.wd3x"; return d; }
+      if (strcmp(force, "v10.wskct") == 0) { d = variant3v10<4, 0, 0, (1 << 21), 3>(); d.name = "v10.wskct"; return d; }
+      if (strcmp(force, "v10.wskba") == 0) { d = variant3v10<4, 0, 0, (1 << 22), 3>(); d.name = "v10.wskba"; return d; }
+      if (strcmp(force, "v10.wskab") == 0) { d = variant3v10<4, 0, 0, (1 << 23), 3>(); d.name = "v10.wskab"; return d; }
+      if (strcmp(force, "v10.wskcx") == 0) { d = variant3v10<4, 0, 0, (1 << 24), 3>(); d.name = "v10.wskcx"; return d; }
+      if (strcmp(force, "v10.wk1") == 0) { d = variant3v10<4, 0, 0, (1 << 27), 3>(); d.name = "v10.wk1"; return d; }
+      if (strcmp(force, "v10.wpk1") == 0) { d = variant3v10<4, 0, 0, (1 << 27) | (1 << 25), 3>(); d.name = "v10.wpk1"; return d; }
+      if (strcmp(force, "v10.wk2") == 0) { d = variant3v10<4, 0, 0, (2 << 27), 3>(); d.name = "v10.wk2"; return d; }
+      if (strcmp(force, "v10.wpk2") == 0) { d = variant3v10<4, 0, 0, (2 << 27) | (1 << 25), 3>(); d.name = "v10.wpk2"; return d; }
+      if (strcmp(force, "v10.wk3") == 0) { d = variant3v10<4, 0, 0, (3 << 27), 3>(); d.name = "v10.wk3"; return d; }
+      if (strcmp(force, "v10.wpk3") == 0) { d = variant3v10<4, 0, 0, (3 << 27) | (1 << 25), 3>(); d.name = "v10.wpk3"; return d; }
       if (strcmp(force, "v10.d2") == 0) { d = variant3v10<4, 2>(); d.name = "v10.d2"; return d; }
       if (strcmp(force, "v5.r2") == 0) { d = variant3v5<4, 0, 2>(); d.name = "v5.r2"; return d; }
       if (strcmp(force, "v5.r1d1") == 0) { d = variant3v5<4, 1, 1>(); d.name = "v5.r1d1"; return d; }

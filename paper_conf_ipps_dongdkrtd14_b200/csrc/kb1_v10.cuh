@@ -90,7 +90,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4, PWG = OPT & 8, V16 = OPT & 16;
   constexpr bool NOXV = OPT & 32;   // timing diagnostic only (wrong results): no x / v gather
   constexpr bool CLK = !(OPT & 4096);   // per-zone clock64 accounting (BLAST_CF_PROFILE); bit 12 compiles it out
-  constexpr int EIG = (OPT & 8192) ? 1 : (OPT & 32768) ? 2 : 0;   // bits 13 / 15: branchy / warp-uniform shortcut of the eigenpair
+  constexpr int EIG = (OPT & 8192) ? 1 : (OPT & 32768) ? 2 : (OPT & 524288) ? 3 : (OPT & 2097152) ? 4 : 0;   // bit 19: diagnostic, no complement   // bits 13 / 15: branchy / warp-uniform shortcut of the eigenpair
   // bit 14 (RHOPW): rho0|J0| is not staged by the contraction warps (512 of their ~1340 cp.async per zone);
   // the point warps prefetch zone i+1's into L2 while they work on zone i and load their two values directly
   constexpr bool RHOPW = OPT & 16384;
@@ -98,6 +98,21 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   // exact dt of the candidates comes from the J^T J the evaluation kept: point a's S is not live across point b
   constexpr bool EARLYS = OPT & 65536;
   constexpr bool SPREAD = OPT & 64;   // the 6 P^3 node-field copies spread over all contraction threads
+  // bits 17 / 18 (timing diagnostics, wrong dt by design): the exact dt of FILTER 2 never / always evaluated
+  // bit 25 (PCT): the POINT warps run the back stage C^T themselves, on DMMA straight from the S values in their
+  // registers -- lane l's two points (q0 = l % 4 and l % 4 + 4, q1 = l / 4, q2 = warp) are exactly the B fragments
+  // of the m8n8k4 tile (k = q0, n = q1) for k-steps 0 and 1 -- and store Y[cd][a0][q1] into their own warp's
+  // rows of the JS buffer (rows col = 8 q2 .. 8 q2 + 7, which only this warp reads); S is never stored and the
+  // contraction warps' back pass starts at B^T
+  // bit 26 (PCTH): the point warps contract fields cd = 0..4 that way, the contraction warps the rest (5..9), also
+  // writing Y into the JS rows (a warp's tile = one q2 row block, read and overwritten by that warp alone)
+  constexpr int NPC = (OPT & (1 << 25)) ? 10 : (OPT & (1 << 26)) ? 5 : 0;   // fields the point warps contract
+  constexpr bool PCT = NPC > 0;
+  constexpr unsigned KSLEEP = ((OPT >> 27) & 3) * 200;   // bits 27-28: timing experiment, contraction warps sleep 200-600 ns   // Y[cd][a0][col] lives in the JS buffer (plane cd, slot q2 * N^2 + a0 * N + q1)
+  constexpr bool NOCV = OPT & 1048576;
+  // bits 21-24 (timing diagnostics, wrong): skip the contraction stage C^T / B^T + A^T / forward A + B / forward C_x
+  constexpr bool SKCT = OPT & (1 << 21), SKBA = OPT & (1 << 22), SKAB = OPT & (1 << 23), SKCX = OPT & (1 << 24);   // bit 20 (timing diagnostic, wrong): no stage C of the velocity fields
+  constexpr int DTX = (OPT & 131072) ? 1 : (OPT & 262144) ? 2 : 0;
   static_assert(!V16 || (Dm::T3 % 2 == 0 && Dm::N3 % 2 == 0 && Dm::XE_E % 2 == 0 && (Dm::OFF_XE + Dm::XE_E) % 2 == 0 &&
                          (Dm::OFF_UV + Dm::O_R) % 2 == 0 && Dm::UVBUF % 2 == 0), "16-byte copies need 16-byte alignment");
   static_assert(!(PWG && (BULK || LATE)), "PWG replaces the contraction warps' gather");
@@ -210,7 +225,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     {
     const int r0_ = kt;
 #pragma unroll
-    for (int blk = 0; blk < (6 * P2 + T2 + NKW - 1) / NKW; ++blk) {
+    for (int blk = 0; blk < (SKAB ? 0 : (6 * P2 + T2 + NKW - 1) / NKW); ++blk) {
       const int r = r0_ + blk * NKW;
       const CTZ<K> C{zc * (blk + 1)};
       if (r < 6 * P2 + T2) {
@@ -254,7 +269,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     constexpr int NB = 6 * N * P, NU = N * T;
     constexpr bool bal = BAL && NKW > NB && NU <= 2 * (NKW - NB) && (NB + NU + NKW - 1) / NKW == 2;
 #pragma unroll
-    for (int blk = 0; blk < (6 * N * P + N * T + NKW - 1) / NKW; ++blk) {
+    for (int blk = 0; blk < (SKAB ? 0 : (6 * N * P + N * T + NKW - 1) / NKW); ++blk) {
       const int r = (bal && blk == 1) ? (r0_ >= NB ? NKW + r0_ - NB : NB + NU) : r0_ + blk * NKW;
       const CTZ<K> C{zc * (blk + 1)};
       if (r < 6 * N * P + N * T) {
@@ -300,7 +315,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     {
     const int r0_ = opaque_tid() - NPW;
 #pragma unroll
-    for (int blk = 0; blk < (9 * N2 + NKW - 1) / NKW; ++blk) {
+    for (int blk = 0; blk < (SKCX ? 0 : (9 * N2 + NKW - 1) / NKW); ++blk) {
       const int r = r0_ + blk * NKW;
       const CTZ<K> C{zc * (blk + 1)};
       if (r < 9 * N2) {
@@ -343,15 +358,15 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       fPt[s] = tfrag<true>(tPhi, T, N, T, lr, 4 * s + lc);
     }
     double *Wr = sWk;
-    {   // C^T: each warp takes one column tile (col = q2*N + q1), five matrices at a time
+    if (NPC < 10) {   // C^T: each warp takes one column tile (col = q2*N + q1), five matrices at a time
       constexpr int NTL = (N2 + 7) / 8;
-      for (int tl = kwarp; tl < NTL; tl += NKWW) {
+      for (int tl = kwarp; tl < (SKCT ? 0 : NTL); tl += NKWW) {
         const int colb = min(tl * 8 + lr, N2 - 1);
         int soff[KS_N];   // swizzled slot of this lane's q0 = 4 s + lc in row colb (kb1_v6.cuh js_idx), once per tile
 #pragma unroll
         for (int s = 0; s < KS_N; ++s) soff[s] = js_idx(colb, min(4 * s + lc, N - 1));
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
+        for (int h = NPC / 5; h < 2; ++h) {
           double sv[5][KS_N];
 #pragma unroll
           for (int c5 = 0; c5 < 5; ++c5)
@@ -373,20 +388,24 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
 #pragma unroll
               for (int c5 = 0; c5 < 5; ++c5) {
                 const int cd = h * 5 + c5;
+                if (PCT) {   // in place over this warp's own S rows (all its loads precede the DMMAs)
+                  if (lr < (cd == 9 ? T : P)) const_cast<double *>(sb)[cd * N3 + tl * N2 + lr * N + 2 * lc + i] = d[c5][i];
+                } else {
                 if (cd < 9 && lr < P) Wr[Dm::O_Y + (cd * P + lr) * Dm::YS + col] = d[c5][i];
                 if (cd == 9 && lr < T) Wr[Dm::O_YE + lr * Dm::YS + col] = d[c5][i];
+                }
               }
             }
           }
         }
       }
     }
-    kw_bar<NKW>();
+    if (NPC < 10) kw_bar<NKW>();
     kstamp(4);
     mid();
     {   // B^T
       constexpr int NC = N * P, NTL = (NC + 7) / 8, NJ = 3 * NTL, JPWT = (NJ + NKWW - 1) / NKWW, JPW = JPWT < KWCH ? JPWT : KWCH;
-      for (int t0 = 0; t0 < JPWT; t0 += JPW) {
+      for (int t0 = 0; t0 < (SKBA ? 0 : JPWT); t0 += JPW) {
         double y[JPW][3][KS_N];
 #pragma unroll
         for (int t = 0; t < JPW; ++t) {
@@ -394,6 +413,16 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
           const int c = j / NTL, tl = j - c * NTL;
           const int nb = min(tl * 8 + lr, NC - 1);
           const int q2b = nb / P, a0b = nb - q2b * P;
+          if (PCT) {   // Y[cd][a0][q1] of column block q2 at JS plane cd, row block q2, slot a0 * 8 + q1
+            const double *Yb = sb + (c * 3) * N3 + q2b * N2 + a0b * N;
+#pragma unroll
+            for (int s = 0; s < KS_N; ++s) {
+              const int q1 = min(4 * s + lc, N - 1);
+              y[t][0][s] = Yb[q1];
+              y[t][1][s] = Yb[N3 + q1];
+              y[t][2][s] = Yb[2 * N3 + q1];
+            }
+          } else {
           const double *Yb = Wr + Dm::O_Y + (c * 3 * P + a0b) * Dm::YS + q2b * N;
 #pragma unroll
           for (int s = 0; s < KS_N; ++s) {
@@ -401,6 +430,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
             y[t][0][s] = Yb[q1];
             y[t][1][s] = Yb[P * Dm::YS + q1];
             y[t][2][s] = Yb[2 * P * Dm::YS + q1];
+          }
           }
         }
         double zb[JPW][2], zg[JPW][2];
@@ -435,7 +465,9 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
         const int q2b = nb / T, j0b = nb - q2b * T;
         double d0 = 0.0, d1 = 0.0;
 #pragma unroll
-        for (int s = 0; s < KS_N; ++s) dmma(d0, d1, fPt[s], Wr[Dm::O_YE + j0b * Dm::YS + q2b * N + min(4 * s + lc, N - 1)]);
+        for (int s = 0; s < KS_N; ++s)
+          dmma(d0, d1, fPt[s], PCT ? sb[9 * N3 + q2b * N2 + j0b * N + min(4 * s + lc, N - 1)]
+                                   : Wr[Dm::O_YE + j0b * Dm::YS + q2b * N + min(4 * s + lc, N - 1)]);
 #pragma unroll
         for (int i = 0; i < 2; ++i) {
           const int n = te * 8 + 2 * lc + i;
@@ -450,7 +482,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     kstamp(5);
     {   // A^T -> global F_z.1 (zone-local) and F^T v
       constexpr int NTL = (P2 + 7) / 8, NJ = 3 * NTL, JPWT = (NJ + NKWW - 1) / NKWW, JPW = JPWT < KWCH ? JPWT : KWCH;
-      for (int t0 = 0; t0 < JPWT; t0 += JPW) {
+      for (int t0 = 0; t0 < (SKBA ? 0 : JPWT); t0 += JPW) {
         double zv[JPW][2][KS_N];
 #pragma unroll
         for (int t = 0; t < JPW; ++t) {
@@ -522,7 +554,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
 #pragma unroll
     for (int i = 0; i < 9; ++i) { ga[i] = 0.0; gb[i] = 0.0; }
 #pragma unroll
-    for (int a0 = 0; a0 < P; ++a0) {
+    for (int a0 = 0; a0 < (NOCV ? 1 : P); ++a0) {
       const double ba = tB[q0a * P + a0], gga = tG[q0a * P + a0];
       const double bb = tB[(q0a + NH) * P + a0], ggb = tG[(q0a + NH) * P + a0];
 #pragma unroll
@@ -568,7 +600,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     } else if (VMODE == 3 && a.ph.use_visc && a.ph.use_vort) {   // both points one straight-line block, one vote
       point_eval3<2, 1, EIG>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best);
       point_eval3<2, 1, EIG>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best);
-      if (__any_sync(0xffffffffu, oa.cand || ob.cand)) {   // J is still in the JS buffer (S is written below)
+      if (DTX != 1 && (DTX == 2 || __any_sync(0xffffffffu, oa.cand || ob.cand))) {   // J is still in the JS buffer (S is written below)
         double Jr[3][3];
 #pragma unroll
         for (int cd = 0; cd < 9; ++cd) Jr[cd / 3][cd % 3] = jb[cd * N3 + sa];
@@ -591,7 +623,38 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       if ((threadIdx.x & 31) == 0 && mi > best)
         atomicMax(reinterpret_cast<unsigned long long *>(sRed + 8), (unsigned long long)__double_as_longlong(mi));
     }
-    if (!(EARLYS && VMODE == 3 && a.ph.use_visc && a.ph.use_vort)) {
+    if (DIAG == 3) {   // keep S live without overwriting J (a store that never happens)
+      double acc = oa.P + ob.P;
+#pragma unroll
+      for (int cd = 0; cd < 9; ++cd) acc += oa.S[cd / 3][cd % 3] + ob.S[cd / 3][cd % 3];
+      if (acc == 1.2345e300) jb[Dm::O_PQ + sa] = acc;
+    } else if (PCT) {
+      static_assert(N == 8 && P <= 8 && T <= 8 && NPW == 256, "PCT: one m8n8k4 tile per (warp, field), k-steps = q0 halves");
+      const int ln = tid & 31, lr = ln >> 2, lc = ln & 3;   // lr = q1, lc = q0a (pr = tid)
+      // A fragments: table^T[a = lr][q0 = 4 s + lc] (rows a >= P / T are zero)
+      const double fb0 = lr < P ? tB[lc * P + lr] : 0.0, fb1 = lr < P ? tB[(lc + 4) * P + lr] : 0.0;
+      const double fg0 = lr < P ? tG[lc * P + lr] : 0.0, fg1 = lr < P ? tG[(lc + 4) * P + lr] : 0.0;
+      const double fp0 = lr < T ? tPhi[lc * T + lr] : 0.0, fp1 = lr < T ? tPhi[(lc + 4) * T + lr] : 0.0;
+      __syncwarp();   // every lane's J (re)reads of this warp's rows precede the Y stores over them
+      double *yw = jb + q2 * N2 + lr * N + 2 * lc;
+#pragma unroll
+      for (int cd = 0; cd < NPC; ++cd) {
+        double d0 = 0.0, d1 = 0.0;
+        const double sa_ = cd < 9 ? oa.S[cd / 3][cd % 3] : oa.P, sb_ = cd < 9 ? ob.S[cd / 3][cd % 3] : ob.P;
+        dmma(d0, d1, cd == 9 ? fp0 : (cd % 3 == 0 ? fg0 : fb0), sa_);
+        dmma(d0, d1, cd == 9 ? fp1 : (cd % 3 == 0 ? fg1 : fb1), sb_);
+        if (lr < (cd == 9 ? T : P)) sts_f64x2(yw + cd * N3, d0, d1);
+      }
+#pragma unroll
+      for (int cd = NPC; cd < 9; ++cd) {   // the contraction warps' fields: S in place over J
+        jb[cd * N3 + sa] = oa.S[cd / 3][cd % 3];
+        jb[cd * N3 + sbi] = ob.S[cd / 3][cd % 3];
+      }
+      if (NPC < 10) {
+        jb[Dm::O_PQ + sa] = oa.P;
+        jb[Dm::O_PQ + sbi] = ob.P;
+      }
+    } else if (!(EARLYS && VMODE == 3 && a.ph.use_visc && a.ph.use_vort)) {
 #pragma unroll
       for (int cd = 0; cd < 9; ++cd) {     // in place over J: only this thread touches slots sa, sbi
         jb[cd * N3 + sa] = oa.S[cd / 3][cd % 3];
@@ -647,7 +710,9 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
         kw_load_id(i + 2);
         cp_async_commit();
       };
-      const bool back = i >= 1 && DIAG != 1;
+      // DIAG 3 (timing only): the point warps alone on valid data -- zones 0 and 1 are formed once, nothing else
+      const bool back = i >= 1 && DIAG != 1 && DIAG != 3;
+      if (KSLEEP > 0 && back) __nanosleep(KSLEEP);   // timing experiment: let the point warps' stage C_v start alone
       if (!PWG && !(LATE && back)) issue();
       kstamp(3);
       const int zc = a.zero * itc;   // 0, but loop-variant and uniform
@@ -660,7 +725,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       }
       kw_bar<NKW>();
       kstamp(7);
-      if (i + 1 < nz && DIAG != 1)
+      if (i + 1 < nz && DIAG != 1 && (DIAG != 3 || i + 1 < 2))
         kw_forward(sUV + ((i + 1) & 1) * Dm::UVBUF, sJS + ((i + 1) & 1) * Dm::JSBUF, sJ + ((i + 1) & 1) * 10, zc + a.zero,
                    PWG ? sXEb[(i + 1) & 1] : sXE);
       if (CLK) t_work += clock64() - t0;
