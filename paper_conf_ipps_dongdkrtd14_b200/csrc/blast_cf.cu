@@ -197,7 +197,6 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
         //  won the autotuner are no longer instantiated; DESIGN.md §10 keeps their measurements)
         add(variant3v10<4, 0, 0, 0, 3>(), "v10.w");
         add(variant3v10<4, 0, 0, (1 << 25), 3>(), "v10.wp");
-        add(variant3v10<4, 0, 0, (1 << 26), 3>(), "v10.wph");
         add(variant3v10<4, 0, 0, 0, 2>(), "v10.v"); add(variant3v5<4, 0, 1>(), "v5.r1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;

@@ -82,7 +82,7 @@ constexpr int v10_smem_bytes() {   // OPT bit 10: PADU's extra 2872 doubles, unu
   return (V10Dims<K, (OPT & 128) != 0, (OPT & 640) != 0, (OPT & 8) || !(OPT & 2048)>::TOTAL + ((OPT & 1024) ? 2872 : 0)) * 8;
 }
 
-template <int K, int DIAG = 0, int MODE = 0, int OPT = 0, int VMODE = 0>
+template <int K, int DIAG = 0, int MODE = 0, int OPT = 0, int VMODE_ = 0>
 __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB1Args a) {
   using Dm = V10Dims<K, (OPT & 128) != 0, (OPT & 640) != 0, (OPT & 8) || !(OPT & 2048)>;   // bit 11: no XEB   // OPT bit 9 (PADE): the UE padding alone
   constexpr int UQ = Dm::UQ, UQ1 = Dm::UQ1, UM = Dm::UM, UQE = Dm::UQE;
@@ -90,13 +90,18 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4, PWG = OPT & 8, V16 = OPT & 16;
   constexpr bool NOXV = OPT & 32;   // timing diagnostic only (wrong results): no x / v gather
   constexpr bool CLK = !(OPT & 4096);   // per-zone clock64 accounting (BLAST_CF_PROFILE); bit 12 compiles it out
-  constexpr int EIG = (OPT & 8192) ? 1 : (OPT & 32768) ? 2 : (OPT & 524288) ? 3 : (OPT & 2097152) ? 4 : 0;   // bit 19: diagnostic, no complement   // bits 13 / 15: branchy / warp-uniform shortcut of the eigenpair
+  constexpr int EIG = (OPT & 8192) ? 1 : (OPT & 32768) ? 2 : (OPT & 524288) ? 3 : (OPT & 2097152) ? 4 : (OPT & (1 << 30)) ? 5 : 0;   // bit 30: the shorter-chain eigenpair   // bit 19: diagnostic, no complement   // bits 13 / 15: branchy / warp-uniform shortcut of the eigenpair
   // bit 14 (RHOPW): rho0|J0| is not staged by the contraction warps (512 of their ~1340 cp.async per zone);
   // the point warps prefetch zone i+1's into L2 while they work on zone i and load their two values directly
   constexpr bool RHOPW = OPT & 16384;
   // bit 16 (EARLYS): each point's S, P go to the JS buffer right after its evaluation (its J is dead), and the
   // exact dt of the candidates comes from the J^T J the evaluation kept: point a's S is not live across point b
   constexpr bool EARLYS = OPT & 65536;
+  // VMODE_ bits 0-1: the point evaluation's switch mode; bits 2+: more options (OPT's bits are used up)
+  constexpr int VMODE = VMODE_ & 3;
+  // VMODE_ bit 2 (DCT): stage C^T on DFMA (v6's form: one (row c, col) item per contraction thread, constant-bank
+  // tables) instead of DMMA -- 2-cycle pipe quanta next to the point warps' DFMAs instead of 16-cycle DMMA tiles
+  constexpr bool DCT = VMODE_ & 4;
   constexpr bool SPREAD = OPT & 64;   // the 6 P^3 node-field copies spread over all contraction threads
   // bits 17 / 18 (timing diagnostics, wrong dt by design): the exact dt of FILTER 2 never / always evaluated
   // bit 25 (PCT): the POINT warps run the back stage C^T themselves, on DMMA straight from the S values in their
@@ -108,6 +113,14 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   // writing Y into the JS rows (a warp's tile = one q2 row block, read and overwritten by that warp alone)
   constexpr int NPC = (OPT & (1 << 25)) ? 10 : (OPT & (1 << 26)) ? 5 : 0;   // fields the point warps contract
   constexpr bool PCT = NPC > 0;
+  // bit 29 (FF, needs PCT): the contraction warps run zone i+1's forward stages A, B FIRST, then zone i-1's B^T,
+  // then C_x(i+1) and A^T(i-1): no DMMA burst at the start of a period (where the point warps' stage C_v and J
+  // loads are).  Z / ZE move below UX (over the dead T), the node gather runs two zones ahead into the two XE
+  // buffers, rho0|J0| one zone ahead, and the contraction warps' cp.async wait moves to the end of the period.
+  constexpr bool FF = OPT & (1 << 29);
+  static_assert(!FF || (PCT && !PWG && !BULK && !LATE && !RHOPW && !SPREAD && !V16), "FF: PCT layout, plain gather");
+  constexpr int O_Z = FF ? 0 : Dm::O_Z, O_ZE = FF ? 6 * Dm::N * Dm::P2 : Dm::O_ZE;
+  static_assert(!FF || 6 * Dm::N * Dm::P2 + Dm::N * Dm::T2 <= Dm::O_UX, "FF: Z / ZE must stay below UX");
   constexpr unsigned KSLEEP = ((OPT >> 27) & 3) * 200;   // bits 27-28: timing experiment, contraction warps sleep 200-600 ns   // Y[cd][a0][col] lives in the JS buffer (plane cd, slot q2 * N^2 + a0 * N + q1)
   constexpr bool NOCV = OPT & 1048576;
   // bits 21-24 (timing diagnostics, wrong): skip the contraction stage C^T / B^T + A^T / forward A + B / forward C_x
@@ -217,10 +230,12 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   auto kw_wait_bulk = [&](int64_t i) {
     if (BULK && i < nz) mbar_wait(sMB + (i & 1), (unsigned)((i >> 1) & 1));
   };
-  auto kw_forward = [&](double *ub, double *jb, double *js, int zc, const double *xe) {
+  // part: 0 = stages A, B, C_x; 1 = A, B only; 2 = C_x only (FF)
+  auto kw_forward = [&](double *ub, double *jb, double *js, int zc, const double *xe, int part = 0) {
     const int kt = opaque_tid() - NPW;
-    if (kt < 10) js[kt] = xe[Dm::XE_J + kt];
     double *Tr = sWk, *UX = sWk + Dm::O_UX;
+    if (part != 2) {
+    if (kt < 10) js[kt] = xe[Dm::XE_J + kt];
     // stage A: a2 -> q2 (T_B, T_G of the 6 fields; TE of e)
     {
     const int r0_ = kt;
@@ -311,6 +326,8 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     }}}
     kw_bar<NKW>();
     kstamp(9);
+    }
+    if (part == 1) return;
     // stage C (position fields): J[c][m](col, q0) = sum_a0 M_m[q0][a0] UX[c][m][col][a0] -> JS (swizzled)
     {
     const int r0_ = opaque_tid() - NPW;
@@ -348,7 +365,8 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     kstamp(10);
   };
   // back stages C^T, B^T, A^T of zone z from the JS buffer sb (S[9][N^3], Pq[N^3])
-  auto kw_back = [&](const double *sb, int64_t z, int, auto &&mid) {
+  // part: 0 = all back stages; 1 = C^T, B^T; 2 = A^T only (FF)
+  auto kw_back = [&](const double *sb, int64_t z, int zc, auto &&mid, int part = 0) {
     const int ktid = opaque_tid() - NPW, kwarp = ktid >> 5, lr = (ktid & 31) >> 2, lc = ktid & 3;
     double fBt[KS_N], fGt[KS_N], fPt[KS_N];
 #pragma unroll
@@ -358,6 +376,42 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       fPt[s] = tfrag<true>(tPhi, T, N, T, lr, 4 * s + lc);
     }
     double *Wr = sWk;
+    if (part != 2) {
+    if (DCT) {   // C^T on DFMA: q0 -> a0 for the 9 S components (3 items per col) and Pq
+      static_assert(!DCT || NPC == 0, "DCT: S in the JS buffer");
+      const int r = opaque_tid() - NPW;
+      const CTZ<K> C{zc};
+      if (r < 4 * N2) {
+        const int c = r / N2, col = r - c * N2;   // warp-uniform c
+        if (c < 3) {
+#pragma unroll
+          for (int d = 0; d < 3; ++d) {   // one S component at a time (register budget of the contraction warps)
+            double sv[N];
+            const double *bd = sb + (c * 3 + d) * N3;
+#pragma unroll
+            for (int pq = 0; pq < N / 2; ++pq) lds_f64x2(bd + js_idx(col, 2 * pq), sv[2 * pq], sv[2 * pq + 1]);
+#pragma unroll
+            for (int a0 = 0; a0 < P; ++a0) {
+              double yv = 0.0;
+#pragma unroll
+              for (int q0 = 0; q0 < N; ++q0) yv = fma(d == 0 ? C.G(q0, a0) : C.B(q0, a0), sv[q0], yv);
+              Wr[Dm::O_Y + ((c * 3 + d) * P + a0) * Dm::YS + col] = yv;
+            }
+          }
+        } else {
+          double pv[N];
+#pragma unroll
+          for (int pq = 0; pq < N / 2; ++pq) lds_f64x2(sb + Dm::O_PQ + js_idx(col, 2 * pq), pv[2 * pq], pv[2 * pq + 1]);
+#pragma unroll
+          for (int j0 = 0; j0 < T; ++j0) {
+            double yv = 0.0;
+#pragma unroll
+            for (int q0 = 0; q0 < N; ++q0) yv = fma(C.Phi(q0, j0), pv[q0], yv);
+            Wr[Dm::O_YE + j0 * Dm::YS + col] = yv;
+          }
+        }
+      }
+    } else
     if (NPC < 10) {   // C^T: each warp takes one column tile (col = q2*N + q1), five matrices at a time
       constexpr int NTL = (N2 + 7) / 8;
       for (int tl = kwarp; tl < (SKCT ? 0 : NTL); tl += NKWW) {
@@ -453,8 +507,8 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
             const int n = tl * 8 + 2 * lc + i;
             if (j < NJ && lr < P && n < NC) {
               const int q2 = n / P, a0 = n - q2 * P;
-              Wr[Dm::O_Z + ((c * 2 + 0) * N + q2) * P2 + lr * P + a0] = zb[t][i];
-              Wr[Dm::O_Z + ((c * 2 + 1) * N + q2) * P2 + lr * P + a0] = zg[t][i];
+              Wr[O_Z + ((c * 2 + 0) * N + q2) * P2 + lr * P + a0] = zb[t][i];
+              Wr[O_Z + ((c * 2 + 1) * N + q2) * P2 + lr * P + a0] = zg[t][i];
             }
           }
         }
@@ -473,13 +527,15 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
           const int n = te * 8 + 2 * lc + i;
           if (lr < T && n < NCE) {
             const int q2 = n / T, j0 = n - q2 * T;
-            Wr[Dm::O_ZE + q2 * T2 + lr * T + j0] = i ? d1 : d0;
+            Wr[O_ZE + q2 * T2 + lr * T + j0] = i ? d1 : d0;
           }
         }
       }
     }
     kw_bar<NKW>();
     kstamp(5);
+    }
+    if (part == 1) return;
     {   // A^T -> global F_z.1 (zone-local) and F^T v
       constexpr int NTL = (P2 + 7) / 8, NJ = 3 * NTL, JPWT = (NJ + NKWW - 1) / NKWW, JPW = JPWT < KWCH ? JPWT : KWCH;
       for (int t0 = 0; t0 < (SKBA ? 0 : JPWT); t0 += JPW) {
@@ -489,7 +545,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
           const int j = min(kwarp + (t0 + t) * NKWW, NJ - 1);
           const int c = j / NTL, tl = j - c * NTL;
           const int nb = min(tl * 8 + lr, P2 - 1);
-          const double *Zb = Wr + Dm::O_Z + c * 2 * N * P2 + nb;
+          const double *Zb = Wr + O_Z + c * 2 * N * P2 + nb;
 #pragma unroll
           for (int s = 0; s < KS_N; ++s) {
             const int q2 = min(4 * s + lc, N - 1);
@@ -525,7 +581,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
         const int nb = min(te * 8 + lr, T2 - 1);
         double d0 = 0.0, d1 = 0.0;
 #pragma unroll
-        for (int s = 0; s < KS_N; ++s) dmma(d0, d1, fPt[s], Wr[Dm::O_ZE + min(4 * s + lc, N - 1) * T2 + nb]);
+        for (int s = 0; s < KS_N; ++s) dmma(d0, d1, fPt[s], Wr[O_ZE + min(4 * s + lc, N - 1) * T2 + nb]);
         if (lr < T) {
 #pragma unroll
           for (int i = 0; i < 2; ++i) {
@@ -684,6 +740,71 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       mbar_init(sMB, 1);
       mbar_init(sMB + 1, 1);
       asm volatile("fence.mbarrier_init.release.cluster;\nfence.proxy.async.shared::cta;\n" ::: "memory");
+    }
+    if (FF) {   // node gather of zone zi into XEb[zi & 1]; rho0|J0| of zone zr into UV[zr & 1]
+      auto ff_nodes = [&](int64_t zi) {
+        if (zi >= nz) return;
+        const int64_t z = zone_of(zi);
+        double *xe = sXEb[zi & 1];
+        if (ktid < P3) {
+          const int64_t node = sID[(zi & 1) * P3 + ktid];
+#pragma unroll
+          for (int c = 0; c < 3; ++c) {
+            cp_async8(xe + Dm::XE_X + c * P3 + ktid, a.x + c * nn + node, true);
+            cp_async8(xe + Dm::XE_X + (3 + c) * P3 + ktid, a.v + c * nn + node, true);
+          }
+        }
+        for (int r = ktid; r < T3 + 10; r += NKW) {
+          const double *src = r < T3 ? a.e + z * T3 + r : r < T3 + 9 ? a.J0inv + z * 9 + (r - T3) : a.zone_gamma + z;
+          cp_async8(xe + Dm::XE_E + r, src, true);
+        }
+      };
+      auto ff_rho = [&](int64_t zr) {
+        if (zr >= nz) return;
+        double *R = sUV + (zr & 1) * Dm::UVBUF + Dm::O_R;
+        const int64_t z = zone_of(zr);
+        for (int r = ktid; r < N3; r += NKW) cp_async8(R + r, a.rho0detJ0 + z * N3 + r, true);
+      };
+      kw_load_id(0);
+      kw_load_id(1);
+      cp_async_commit();
+      cp_async_wait<0>();
+      kw_bar<NKW>();
+      ff_nodes(0);
+      ff_rho(0);
+      ff_nodes(1);
+      kw_load_id(2);
+      cp_async_commit();
+      cp_async_wait<0>();
+      kw_bar<NKW>();
+      if (nz > 0) kw_forward(sUV, sJS, sJ, a.zero, sXEb[0]);
+      cta_bar_div<Cfg::NTH>();
+      long long t_work = 0;
+      int itc = 2;
+      for (int64_t i = 0; i <= nz; ++i, ++itc) {
+        const long long t0 = CLK ? clock64() : 0;
+        ff_nodes(i + 2);
+        ff_rho(i + 1);
+        kw_load_id(i + 3);
+        cp_async_commit();
+        kstamp(3);
+        const int zc = a.zero * itc;
+        const bool fw = i + 1 < nz, back = i >= 1;
+        double *ub1 = sUV + ((i + 1) & 1) * Dm::UVBUF, *jb1 = sJS + ((i + 1) & 1) * Dm::JSBUF, *js1 = sJ + ((i + 1) & 1) * 10;
+        if (fw) kw_forward(ub1, jb1, js1, zc + a.zero, sXEb[(i + 1) & 1], 1);   // A, B (ends with a KW barrier)
+        if (back) kw_back(sJS + ((i - 1) & 1) * Dm::JSBUF, zone_of(i - 1), zc, [] {}, 1);   // B^T (ends with a barrier)
+        if (fw) kw_forward(ub1, jb1, js1, zc + a.zero, sXEb[(i + 1) & 1], 2);   // C_x: J(i+1) over Y(i-1), read by B^T
+        if (back) kw_back(sJS + ((i - 1) & 1) * Dm::JSBUF, zone_of(i - 1), zc, [] {}, 2);   // A^T (+ KW barrier)
+        cp_async_wait<0>();   // zone i+2's nodes, zone i+1's rho0|J0| (read by the point warps next period)
+        if (CLK) t_work += clock64() - t0;
+        cta_bar_div<Cfg::NTH>();
+        kstamp(11);
+      }
+      if (a.prof != nullptr && tid == NPW) {
+        a.prof[blockIdx.x * 16 + 1] = t_work;
+        for (int sl = 3; sl < 12; ++sl) a.prof[blockIdx.x * 16 + sl] = sKP[sl];
+      }
+      return;
     }
     if (PWG) {   // the point warps issue the gathers
       if (nz > 0) mbar_wait(sMB, 0u);
