@@ -93,16 +93,16 @@ void launch2(const KB1Args &a, int grid, cudaStream_t s) {
   using C = KB1Cfg2<K, ZPC>;
   kb1_corner_force_2d<K, ZPC, MINB><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
 }
-template <int K, int ZPC, int MINB, int PPT>
+template <int K, int ZPC, int MINB, int PPT, int EX>
 void launch3v2(const KB1Args &a, int grid, cudaStream_t s) {
   using C = KB1V2Cfg<K, ZPC, PPT>;
-  kb1_v2_3d<K, ZPC, MINB, PPT><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
+  kb1_v2_3d<K, ZPC, MINB, PPT, EX><<<grid, C::NTH, C::SMEM_BYTES, s>>>(a);
 }
-template <int K, int ZPC, int MINB, int PPT = 2>
+template <int K, int ZPC, int MINB, int PPT = 2, int EX = 0>
 KB1Variant variant3v2() {
   using C = KB1V2Cfg<K, ZPC, PPT>;
-  return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3v2<K, ZPC, MINB, PPT>,
-                    (const void *)&kb1_v2_3d<K, ZPC, MINB, PPT>, true, nullptr};
+  return KB1Variant{ZPC, C::NTH, C::SMEM_BYTES, &launch3v2<K, ZPC, MINB, PPT, EX>,
+                    (const void *)&kb1_v2_3d<K, ZPC, MINB, PPT, EX>, true, nullptr};
 }
 template <int K, int ZPC, int MINB>
 void launch3v3(const KB1Args &a, int grid, cudaStream_t s) {
@@ -190,20 +190,22 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
   if (dim == 3) {
     switch (k) {
       case 1: add(variant3v2<1, 32, 2, 1>(), "v2.p1.z32"); add(variant3v2<1, 64, 2>(), "v2.z64"); add(variant3<1, 32, 2>(), "v1.z32"); break;
-      case 2: add(variant3v2<2, 1, 12>(), "v2.z1m12"); add(variant3v2<2, 2, 6>(), "v2.z2m6"); add(variant3v2<2, 2, 4, 1>(), "v2.p1.z2"); add(variant3<2, 16, 2>(), "v1.z16"); break;
+      case 2: add(variant3v2<2, 1, 12, 2, 6>(), "v2.z1m12e"); add(variant3v2<2, 1, 12>(), "v2.z1m12"); add(variant3v2<2, 2, 6>(), "v2.z2m6"); add(variant3v2<2, 2, 4, 1>(), "v2.p1.z2"); add(variant3<2, 16, 2>(), "v1.z16"); break;
       case 3: add(variant3v2<3, 2, 2>(), "v2.z2"); add(variant3v2<3, 1, 2, 1>(), "v2.p1.z1"); add(variant3v3<3, 2, 2>(), "v3.z2"); add(variant3<3, 8, 2>(), "v1.z8"); break;
       case 4:
         // (round 2: the superseded generations v10 (runtime switches), v10.wu, v6, v5, v4.m0/m1, v3.z1 that never
         //  won the autotuner are no longer instantiated; DESIGN.md §10 keeps their measurements)
+        add(variant3v10<4, 0, 0, (1 << 25), 3 | 8>(), "v10.wpx");
         add(variant3v10<4, 0, 0, 0, 3>(), "v10.w");
         add(variant3v10<4, 0, 0, (1 << 25), 3>(), "v10.wp");
+        add(variant3v10<4, 0, 0, 0, 3 | 8>(), "v10.wx");
         add(variant3v10<4, 0, 0, 0, 2>(), "v10.v"); add(variant3v5<4, 0, 1>(), "v5.r1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
       case 6: add(variant3<6, 1, 2>(), "v1.z1m2"); add(variant3<6, 2, 1>(), "v1.z2"); break;
       case 7: add(variant3v8<7, 1>(), "v8"); add(variant3v11<7, 1>(), "v11"); add(variant3<7, 1, 2>(), "v1.z1"); break;
-      case 8: add(variant3v11<8, 2, 83>(), "v11.mbtsi"); add(variant3v11<8, 2, 19>(), "v11.mbts"); add(variant3v11<8, 2, 3>(), "v11.mbt"); add(variant3v11<8, 2, 1>(), "v11.mb"); add(variant3v8<8, 2>(), "v8"); add(variant3v11<8, 2>(), "v11"); add(variant3v8<8, 1>(), "v8.m1"); add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
+      case 8: add(variant3v11<8, 2, 83 | 128>(), "v11.mbtsie"); add(variant3v11<8, 2, 83>(), "v11.mbtsi"); add(variant3v11<8, 2, 19>(), "v11.mbts"); add(variant3v11<8, 2, 3>(), "v11.mbt"); add(variant3v11<8, 2, 1>(), "v11.mb"); add(variant3v8<8, 2>(), "v8"); add(variant3v11<8, 2>(), "v11"); add(variant3v8<8, 1>(), "v8.m1"); add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
     }
   } else {
     switch (k) {
@@ -281,6 +283,14 @@ KB1Variant select_variant(int dim, int k, bool need_point_j0) {
       if (strcmp(force, "v10.wpk2") == 0) { d = variant3v10<4, 0, 0, (2 << 27) | (1 << 25), 3>(); d.name = "v10.wpk2"; return d; }
       if (strcmp(force, "v10.wk3") == 0) { d = variant3v10<4, 0, 0, (3 << 27), 3>(); d.name = "v10.wk3"; return d; }
       if (strcmp(force, "v10.wpk3") == 0) { d = variant3v10<4, 0, 0, (3 << 27) | (1 << 25), 3>(); d.name = "v10.wpk3"; return d; }
+      if (strcmp(force, "v10.wxr4") == 0) { d = variant3v10<4, 0, 4, 0, 3 | 8>(); d.name = "v10.wxr4"; return d; }
+      if (strcmp(force, "v10.wxr3") == 0) { d = variant3v10<4, 0, 3, 0, 3 | 8>(); d.name = "v10.wxr3"; return d; }
+      if (strcmp(force, "v10.wpxr4") == 0) { d = variant3v10<4, 0, 4, (1 << 25), 3 | 8>(); d.name = "v10.wpxr4"; return d; }
+      if (strcmp(force, "v10.wpxk1") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | (1 << 27), 3 | 8>(); d.name = "v10.wpxk1"; return d; }
+      if (strcmp(force, "v10.wpxk2") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | (2 << 27), 3 | 8>(); d.name = "v10.wpxk2"; return d; }
+      if (strcmp(force, "v10.wpxb") == 0) { d = variant3v10<4, 0, 0, (1 << 25), 3 | 8 | 16>(); d.name = "v10.wpxb"; return d; }
+      if (strcmp(force, "v10.wpxd3") == 0) { d = variant3v10<4, 3, 0, (1 << 25), 3 | 8>(); d.name = "v10.wpxd3"; return d; }
+      if (strcmp(force, "v10.wpxd2") == 0) { d = variant3v10<4, 2, 0, (1 << 25), 3 | 8>(); d.name = "v10.wpxd2"; return d; }
       if (strcmp(force, "v10.d2") == 0) { d = variant3v10<4, 2>(); d.name = "v10.d2"; return d; }
       if (strcmp(force, "v5.r2") == 0) { d = variant3v5<4, 0, 2>(); d.name = "v5.r2"; return d; }
       if (strcmp(force, "v5.r1d1") == 0) { d = variant3v5<4, 1, 1>(); d.name = "v5.r1d1"; return d; }

@@ -90,7 +90,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   constexpr bool BULK = OPT & 1, LATE = OPT & 2, BAL = OPT & 4, PWG = OPT & 8, V16 = OPT & 16;
   constexpr bool NOXV = OPT & 32;   // timing diagnostic only (wrong results): no x / v gather
   constexpr bool CLK = !(OPT & 4096);   // per-zone clock64 accounting (BLAST_CF_PROFILE); bit 12 compiles it out
-  constexpr int EIG = (OPT & 8192) ? 1 : (OPT & 32768) ? 2 : (OPT & 524288) ? 3 : (OPT & 2097152) ? 4 : (OPT & (1 << 30)) ? 5 : 0;   // bit 30: the shorter-chain eigenpair   // bit 19: diagnostic, no complement   // bits 13 / 15: branchy / warp-uniform shortcut of the eigenpair
+  constexpr int EIG = (OPT & 8192) ? 1 : (OPT & 32768) ? 2 : (OPT & 524288) ? 3 : (OPT & 2097152) ? 4 : (OPT & (1 << 30)) ? 5 : (VMODE_ & 8) ? 6 : 0;   // bit 30: the shorter-chain eigenpair   // bit 19: diagnostic, no complement   // bits 13 / 15: branchy / warp-uniform shortcut of the eigenpair
   // bit 14 (RHOPW): rho0|J0| is not staged by the contraction warps (512 of their ~1340 cp.async per zone);
   // the point warps prefetch zone i+1's into L2 while they work on zone i and load their two values directly
   constexpr bool RHOPW = OPT & 16384;
@@ -102,6 +102,10 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   // VMODE_ bit 2 (DCT): stage C^T on DFMA (v6's form: one (row c, col) item per contraction thread, constant-bank
   // tables) instead of DMMA -- 2-cycle pipe quanta next to the point warps' DFMAs instead of 16-cycle DMMA tiles
   constexpr bool DCT = VMODE_ & 4;
+  // VMODE_ bit 4 (KWB, needs PCT): the contraction warps compute every point's dt-filter bound (J^T J and
+  // q - sqrt(2/3) |J^T J - q I|_F, pointwise.cuh dt_filter_bound_J) right after stage C_x, into the JS buffer's
+  // tenth plane (free until the point warps' YE stores): ~30 FP64 instructions per point off the point warps
+  constexpr bool KWB = VMODE_ & 16;
   constexpr bool SPREAD = OPT & 64;   // the 6 P^3 node-field copies spread over all contraction threads
   // bits 17 / 18 (timing diagnostics, wrong dt by design): the exact dt of FILTER 2 never / always evaluated
   // bit 25 (PCT): the POINT warps run the back stage C^T themselves, on DMMA straight from the S values in their
@@ -362,6 +366,19 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
 #pragma unroll
       for (int pq = 0; pq < N / 2; ++pq) sts_f64x2(dst + js_idx(col, 2 * pq), o[2 * pq], o[2 * pq + 1]);
     }}}
+    if (KWB) {   // the dt-filter bound of every point of this zone into plane 9 (after all of J is stored)
+      static_assert(!KWB || (PCT && N3 == 2 * NKW), "KWB: two points per contraction thread, plane 9 free (PCT)");
+      kw_bar<NKW>();
+      const int kt2 = opaque_tid() - NPW;
+#pragma unroll 1
+      for (int h = 0; h < 2; ++h) {
+        const int pidx = kt2 + h * NKW, slot = js_idx(pidx >> 3, pidx & 7);
+        double Jr[3][3];
+#pragma unroll
+        for (int cd = 0; cd < 9; ++cd) Jr[cd / 3][cd % 3] = jb[cd * N3 + slot];
+        jb[Dm::O_PQ + slot] = dt_filter_bound_J(Jr);
+      }
+    }
     kstamp(10);
   };
   // back stages C^T, B^T, A^T of zone z from the JS buffer sb (S[9][N^3], Pq[N^3])
@@ -654,8 +671,9 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
         point_dt_exact_m(ob.m, a.ph, ob);
       }
     } else if (VMODE == 3 && a.ph.use_visc && a.ph.use_vort) {   // both points one straight-line block, one vote
-      point_eval3<2, 1, EIG>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best);
-      point_eval3<2, 1, EIG>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best);
+      const double la = KWB ? jb[Dm::O_PQ + sa] : 0.0, lb = KWB ? jb[Dm::O_PQ + sbi] : 0.0;
+      point_eval3<2, 1, EIG, KWB ? 1 : 0>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best, 0xffffffffu, la);
+      point_eval3<2, 1, EIG, KWB ? 1 : 0>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best, 0xffffffffu, lb);
       if (DTX != 1 && (DTX == 2 || __any_sync(0xffffffffu, oa.cand || ob.cand))) {   // J is still in the JS buffer (S is written below)
         double Jr[3][3];
 #pragma unroll
@@ -679,7 +697,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       if ((threadIdx.x & 31) == 0 && mi > best)
         atomicMax(reinterpret_cast<unsigned long long *>(sRed + 8), (unsigned long long)__double_as_longlong(mi));
     }
-    if (DIAG == 3) {   // keep S live without overwriting J (a store that never happens)
+    if (DIAG == 3 && !PCT) {   // keep S live without overwriting J (a store that never happens)
       double acc = oa.P + ob.P;
 #pragma unroll
       for (int cd = 0; cd < 9; ++cd) acc += oa.S[cd / 3][cd % 3] + ob.S[cd / 3][cd % 3];
@@ -692,7 +710,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       const double fg0 = lr < P ? tG[lc * P + lr] : 0.0, fg1 = lr < P ? tG[(lc + 4) * P + lr] : 0.0;
       const double fp0 = lr < T ? tPhi[lc * T + lr] : 0.0, fp1 = lr < T ? tPhi[(lc + 4) * T + lr] : 0.0;
       __syncwarp();   // every lane's J (re)reads of this warp's rows precede the Y stores over them
-      double *yw = jb + q2 * N2 + lr * N + 2 * lc;
+      double *yw = (DIAG == 3 ? sWk : jb) + q2 * N2 + lr * N + 2 * lc;   // DIAG 3: J must survive (timing only)
 #pragma unroll
       for (int cd = 0; cd < NPC; ++cd) {
         double d0 = 0.0, d1 = 0.0;

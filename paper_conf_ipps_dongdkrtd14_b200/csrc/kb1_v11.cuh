@@ -296,7 +296,7 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
         PointOut<3> pt;
         if (FILTER) {
           const double best = sRed[8];
-          point_eval3<true>(Jm, Gv, eq, R, alpha, sJ0[9], sJ0, a.ph, pt, best);
+          point_eval3<true, 0, (MB & 128) ? 6 : 0>(Jm, Gv, eq, R, alpha, sJ0[9], sJ0, a.ph, pt, best);
           double mi = pt.inv;
 #pragma unroll
           for (int s = 16; s > 0; s >>= 1) mi = fmax(mi, __shfl_xor_sync(0xffffffffu, mi, s));

@@ -80,7 +80,8 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int NPEND>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(NPEND)); }
 
-template <int K, int ZPC, int MINB, int PPT = 2>
+// EX = 6: the point evaluation's lean eigen-solve (pointwise.cuh sym3_min_eig_lean, alpha folded into sigma)
+template <int K, int ZPC, int MINB, int PPT = 2, int EX = 0>
 __global__ void __launch_bounds__(KB1V2Cfg<K, ZPC, PPT>::NTH, MINB) kb1_v2_3d(const KB1Args a) {
   using Dm = V2Dims<K>;
   using C = CT<K>;
@@ -303,7 +304,7 @@ __global__ void __launch_bounds__(KB1V2Cfg<K, ZPC, PPT>::NTH, MINB) kb1_v2_3d(co
       {   // dt filter (pointwise.cuh): exact sigma_min(J) only where a point can beat the CTA's best inverse dt
         const unsigned vm = __activemask();
         const double best = sRed[16];
-        point_eval3<true>(Jm, Gv, eq, R, alpha, gamma, J0i, a.ph, o, best, vm);
+        point_eval3<true, 0, EX>(Jm, Gv, eq, R, alpha, gamma, J0i, a.ph, o, best, vm);
         if (active && o.inv > best)
           atomicMax(reinterpret_cast<unsigned long long *>(sRed + 16), (unsigned long long)__double_as_longlong(o.inv));
       }

@@ -285,10 +285,10 @@ def test_multi_material_gamma(orc):
     check(m, s, orc)
 
 
-CANDIDATES = {1: ["v2.p1.z32", "v2.z64", "v1.z32"], 2: ["v2.z1m12", "v2.z2m6", "v2.p1.z2", "v1.z16"],
+CANDIDATES = {1: ["v2.p1.z32", "v2.z64", "v1.z32"], 2: ["v2.z1m12e", "v2.z1m12", "v2.z2m6", "v2.p1.z2", "v1.z16"],
               3: ["v2.z2", "v2.p1.z1", "v3.z2", "v1.z8"],
-              4: ["v10.w", "v10.wp", "v10.v", "v5.r1", "v2.z1", "v1.z4"],
-              7: ["v8", "v11", "v1.z1"], 8: ["v11.mbtsi", "v11.mbts", "v11.mbt", "v11.mb", "v8", "v11", "v8.m1", "v1.z1m2", "v1.z1"]}
+              4: ["v10.wpx", "v10.w", "v10.wp", "v10.wx", "v10.v", "v5.r1", "v2.z1", "v1.z4"],
+              7: ["v8", "v11", "v1.z1"], 8: ["v11.mbtsie", "v11.mbtsi", "v11.mbts", "v11.mbt", "v11.mb", "v8", "v11", "v8.m1", "v1.z1m2", "v1.z1"]}
 
 
 @pytest.mark.parametrize("k,name", [(k, n) for k, ns in CANDIDATES.items() for n in ns])
@@ -340,7 +340,7 @@ def _switch_params(visc, vort):
 
 @pytest.mark.parametrize("visc,vort", SWITCHES)
 @pytest.mark.parametrize("k,name", [(4, n) for n in CANDIDATES[4]] + [(8, n) for n in CANDIDATES[8]] +
-                         [(2, "v2.z1m12"), (3, "v2.z2"), (7, "v8")])
+                         [(2, "v2.z1m12e"), (2, "v2.z1m12"), (3, "v2.z2"), (7, "v8")])
 def test_switches_every_candidate(orc, k, name, visc, vort, monkeypatch):
     """Viscosity / vorticity switches off through every C4 and C5 candidate (the compile-time-switch
     kernels v10.w / v10.v fall back to their runtime-switch branch), on S1 with point-varying rho0|J0|."""

@@ -1,7 +1,7 @@
 #!/bin/bash
 # compute-sanitizer memcheck / racecheck / synccheck / initcheck over the cases of tools/sanitize.py (under gpurun)
 mkdir -p gpurun_out
-out=gpurun_out/r02_sanitizer.txt
+out=gpurun_out/r02s3_sanitizer.txt
 : > $out
 for tool in memcheck synccheck racecheck initcheck; do
   for c in c4 c5 c5v8 c3 c2 integrator host loopback; do
