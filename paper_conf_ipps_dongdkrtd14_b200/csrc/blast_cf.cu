@@ -240,6 +240,21 @@ KB1Variant select_variant(int dim, int k, bool need_point_j0) {
     if (need_point_j0) return c[0];
     // timing diagnostics (wrong results by design; never candidates of the autotuner): compiled only into a
     // -DBLAST_CF_DIAGNOSTICS build, never into the production library
+    if (dim == 3 && k == 2) {
+      KB1Variant d;
+      if (strcmp(force, "v2.p1.z2e") == 0) { d = variant3v2<2, 2, 4, 1, 6>(); d.name = "v2.p1.z2e"; return d; }
+      if (strcmp(force, "v2.p1.z2m5e") == 0) { d = variant3v2<2, 2, 5, 1, 6>(); d.name = "v2.p1.z2m5e"; return d; }
+      if (strcmp(force, "v2.p1.z1m8e") == 0) { d = variant3v2<2, 1, 8, 1, 6>(); d.name = "v2.p1.z1m8e"; return d; }
+      if (strcmp(force, "v2.p1.z1m10e") == 0) { d = variant3v2<2, 1, 10, 1, 6>(); d.name = "v2.p1.z1m10e"; return d; }
+      if (strcmp(force, "v2.z1m13e") == 0) { d = variant3v2<2, 1, 13, 2, 6>(); d.name = "v2.z1m13e"; return d; }
+      if (strcmp(force, "v2.z1m11e") == 0) { d = variant3v2<2, 1, 11, 2, 6>(); d.name = "v2.z1m11e"; return d; }
+    }
+    if (dim == 3 && k == 8) {
+      KB1Variant d;
+      if (strcmp(force, "v11.mbtcie") == 0) { d = variant3v11<8, 2, 83 | 128 | 4>(); d.name = "v11.mbtcie"; return d; }
+      if (strcmp(force, "v11.mbtce") == 0) { d = variant3v11<8, 2, 19 | 128 | 4>(); d.name = "v11.mbtce"; return d; }
+      if (strcmp(force, "v11.mbtse") == 0) { d = variant3v11<8, 2, 19 | 128>(); d.name = "v11.mbtse"; return d; }
+    }
     if (dim == 3 && k == 4) {
       KB1Variant d;
       if (strcmp(force, "v5.d1") == 0) { d = variant3v5<4, 1>(); d.name = "v5.d1"; return d; }
@@ -291,6 +306,10 @@ KB1Variant select_variant(int dim, int k, bool need_point_j0) {
       if (strcmp(force, "v10.wpxb") == 0) { d = variant3v10<4, 0, 0, (1 << 25), 3 | 8 | 16>(); d.name = "v10.wpxb"; return d; }
       if (strcmp(force, "v10.wpxd3") == 0) { d = variant3v10<4, 3, 0, (1 << 25), 3 | 8>(); d.name = "v10.wpxd3"; return d; }
       if (strcmp(force, "v10.wpxd2") == 0) { d = variant3v10<4, 2, 0, (1 << 25), 3 | 8>(); d.name = "v10.wpxd2"; return d; }
+      if (strcmp(force, "v10.wpxncv") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | 1048576, 3 | 8>(); d.name = "v10.wpxncv"; return d; }
+      if (strcmp(force, "v10.wpxnc") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | 524288, 3>(); d.name = "v10.wpxnc"; return d; }
+      if (strcmp(force, "v10.wpxskba") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | (1 << 22), 3 | 8>(); d.name = "v10.wpxskba"; return d; }
+      if (strcmp(force, "v10.wpxd4") == 0) { d = variant3v10<4, 4, 0, (1 << 25), 3 | 8>(); d.name = "v10.wpxd4"; return d; }
       if (strcmp(force, "v10.d2") == 0) { d = variant3v10<4, 2>(); d.name = "v10.d2"; return d; }
       if (strcmp(force, "v5.r2") == 0) { d = variant3v5<4, 0, 2>(); d.name = "v5.r2"; return d; }
       if (strcmp(force, "v5.r1d1") == 0) { d = variant3v5<4, 1, 1>(); d.name = "v5.r1d1"; return d; }
@@ -893,6 +912,7 @@ int blast_cf_create(const blast_cf_mesh *mesh, int order, int dim, const blast_c
     if (cudaEventCreate(&e) != cudaSuccess) return bail(fail(BLAST_CF_ECUDA, "event create"));
   if (getenv("BLAST_CF_PROFILE") && cudaMalloc(&h->d_prof, std::max<int64_t>(h->ncta_cap, 1) * 16 * sizeof(long long)) != cudaSuccess)
     return bail(fail(BLAST_CF_ENOMEM, "profile buffer"));
+  if (h->d_prof) cudaMemset(h->d_prof, 0, std::max<int64_t>(h->ncta_cap, 1) * 16 * sizeof(long long));
   // the uploads above are legacy-stream copies from pageable memory: make sure they have landed before any eval
   // is enqueued on a (possibly non-blocking) user stream
   if (cudaDeviceSynchronize() != cudaSuccess) return bail(fail(BLAST_CF_ECUDA, "create: %s", cudaGetErrorString(cudaGetLastError())));

@@ -615,6 +615,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   // ---------------- PW ----------------
   double dtmin = __longlong_as_double(0x7ff0000000000000LL);
   bool bad = false;
+  long long nvote4 = 0, nexact4 = 0;   // DIAG 4 counters
   const int pr = tid, q0a = pr % NH, q1 = (pr / NH) % N, q2 = pr / (NH * N);
   auto pw_point = [&](const double *ub, const double *js, double *jb, int64_t z) {
     const double gamma = js[9];
@@ -674,7 +675,9 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       const double la = KWB ? jb[Dm::O_PQ + sa] : 0.0, lb = KWB ? jb[Dm::O_PQ + sbi] : 0.0;
       point_eval3<2, 1, EIG, KWB ? 1 : 0>(Ja, Gva, ea, Ra, sW[q0a] * w12, gamma, js, a.ph, oa, best, 0xffffffffu, la);
       point_eval3<2, 1, EIG, KWB ? 1 : 0>(Jb, Gvb, eb, Rb, sW[q0a + NH] * w12, gamma, js, a.ph, ob, best, 0xffffffffu, lb);
-      if (DTX != 1 && (DTX == 2 || __any_sync(0xffffffffu, oa.cand || ob.cand))) {   // J is still in the JS buffer (S is written below)
+      const bool anyc = __any_sync(0xffffffffu, oa.cand || ob.cand);
+      if (DIAG == 4) { nvote4 += 1; nexact4 += anyc ? 1 : 0; }   // DIAG 4 (counting only): how often the exact dt runs
+      if (DTX != 1 && (DTX == 2 || anyc)) {   // J is still in the JS buffer (S is written below)
         double Jr[3][3];
 #pragma unroll
         for (int cd = 0; cd < 9; ++cd) Jr[cd / 3][cd % 3] = jb[cd * N3 + sa];
@@ -941,6 +944,10 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   if (a.prof != nullptr && tid == 0) {
     a.prof[blockIdx.x * 16 + 0] = t_work;
     a.prof[blockIdx.x * 16 + 2] = clock64() - t_all;
+  }
+  if (DIAG == 4 && a.prof != nullptr && (tid & 31) == 0 && tid < NPW) {
+    atomicAdd(reinterpret_cast<unsigned long long *>(a.prof + blockIdx.x * 16 + 12), (unsigned long long)nvote4);
+    atomicAdd(reinterpret_cast<unsigned long long *>(a.prof + blockIdx.x * 16 + 13), (unsigned long long)nexact4);
   }
   if (bad) dtmin = 0.0;
 #pragma unroll
