@@ -197,8 +197,6 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
         //  won the autotuner are no longer instantiated; DESIGN.md §10 keeps their measurements)
         add(variant3v10<4, 0, 0, (1 << 25), 3 | 8>(), "v10.wpx");
         add(variant3v10<4, 0, 0, 0, 3>(), "v10.w");
-        add(variant3v10<4, 0, 0, (1 << 25), 3>(), "v10.wp");
-        add(variant3v10<4, 0, 0, 0, 3 | 8>(), "v10.wx");
         add(variant3v10<4, 0, 0, 0, 2>(), "v10.v"); add(variant3v5<4, 0, 1>(), "v5.r1");
         add(variant3v2<4, 1, 2>(), "v2.z1"); add(variant3<4, 4, 2>(), "v1.z4");
         break;
@@ -310,6 +308,10 @@ KB1Variant select_variant(int dim, int k, bool need_point_j0) {
       if (strcmp(force, "v10.wpxnc") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | 524288, 3>(); d.name = "v10.wpxnc"; return d; }
       if (strcmp(force, "v10.wpxskba") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | (1 << 22), 3 | 8>(); d.name = "v10.wpxskba"; return d; }
       if (strcmp(force, "v10.wpxd4") == 0) { d = variant3v10<4, 4, 0, (1 << 25), 3 | 8>(); d.name = "v10.wpxd4"; return d; }
+      if (strcmp(force, "v10.wpxr3") == 0) { d = variant3v10<4, 0, 3, (1 << 25), 3 | 8>(); d.name = "v10.wpxr3"; return d; }
+      if (strcmp(force, "v10.wpxr1") == 0) { d = variant3v10<4, 0, 1, (1 << 25), 3 | 8>(); d.name = "v10.wpxr1"; return d; }
+      if (strcmp(force, "v10.wp") == 0) { d = variant3v10<4, 0, 0, (1 << 25), 3>(); d.name = "v10.wp"; return d; }
+      if (strcmp(force, "v10.wx") == 0) { d = variant3v10<4, 0, 0, 0, 3 | 8>(); d.name = "v10.wx"; return d; }
       if (strcmp(force, "v10.d2") == 0) { d = variant3v10<4, 2>(); d.name = "v10.d2"; return d; }
       if (strcmp(force, "v5.r2") == 0) { d = variant3v5<4, 0, 2>(); d.name = "v5.r2"; return d; }
       if (strcmp(force, "v5.r1d1") == 0) { d = variant3v5<4, 1, 1>(); d.name = "v5.r1d1"; return d; }
