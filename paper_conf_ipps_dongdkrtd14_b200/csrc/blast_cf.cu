@@ -203,7 +203,7 @@ std::vector<KB1Variant> kb1_candidates(int dim, int k) {
       case 5: add(variant3<5, 2, 2>(), "v1.z2"); break;
       case 6: add(variant3<6, 1, 2>(), "v1.z1m2"); add(variant3<6, 2, 1>(), "v1.z2"); break;
       case 7: add(variant3v8<7, 1>(), "v8"); add(variant3v11<7, 1>(), "v11"); add(variant3<7, 1, 2>(), "v1.z1"); break;
-      case 8: add(variant3v11<8, 2, 83 | 128>(), "v11.mbtsie"); add(variant3v11<8, 2, 83>(), "v11.mbtsi"); add(variant3v11<8, 2, 19>(), "v11.mbts"); add(variant3v11<8, 2, 3>(), "v11.mbt"); add(variant3v11<8, 2, 1>(), "v11.mb"); add(variant3v8<8, 2>(), "v8"); add(variant3v11<8, 2>(), "v11"); add(variant3v8<8, 1>(), "v8.m1"); add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
+      case 8: add(variant3v11<8, 2, 83 | 128 | 256>(), "v11.mbtsiet"); add(variant3v11<8, 2, 83 | 128>(), "v11.mbtsie"); add(variant3v11<8, 2, 83>(), "v11.mbtsi"); add(variant3v11<8, 2, 19>(), "v11.mbts"); add(variant3v11<8, 2, 3>(), "v11.mbt"); add(variant3v11<8, 2, 1>(), "v11.mb"); add(variant3v8<8, 2>(), "v8"); add(variant3v11<8, 2>(), "v11"); add(variant3v8<8, 1>(), "v8.m1"); add(variant3<8, 1, 2>(), "v1.z1m2"); add(variant3<8, 1, 1>(), "v1.z1"); break;
     }
   } else {
     switch (k) {
@@ -312,6 +312,7 @@ KB1Variant select_variant(int dim, int k, bool need_point_j0) {
       if (strcmp(force, "v10.wpxr1") == 0) { d = variant3v10<4, 0, 1, (1 << 25), 3 | 8>(); d.name = "v10.wpxr1"; return d; }
       if (strcmp(force, "v10.wp") == 0) { d = variant3v10<4, 0, 0, (1 << 25), 3>(); d.name = "v10.wp"; return d; }
       if (strcmp(force, "v10.wx") == 0) { d = variant3v10<4, 0, 0, 0, 3 | 8>(); d.name = "v10.wx"; return d; }
+      if (strcmp(force, "v10.wphx") == 0) { d = variant3v10<4, 0, 0, (1 << 26), 3 | 8>(); d.name = "v10.wphx"; return d; }
       if (strcmp(force, "v10.d2") == 0) { d = variant3v10<4, 2>(); d.name = "v10.d2"; return d; }
       if (strcmp(force, "v5.r2") == 0) { d = variant3v5<4, 0, 2>(); d.name = "v5.r2"; return d; }
       if (strcmp(force, "v5.r1d1") == 0) { d = variant3v5<4, 1, 1>(); d.name = "v5.r1d1"; return d; }

@@ -164,9 +164,24 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
         constexpr int NTILE = NB + NG + 1;                          // + one tile of the 8 e lines
         const int lr = lane >> 2, lc = lane & 3;
         static_assert(!MB || 6 * P == 54, "the [a1][108] T layout");
+        // MB bit 8 (TBW): warps 0-4 take the 14 B-table tiles, warps 5-7 the 7 G-table tiles and the Phi tile, so a
+        // warp's A fragments (its table's rows 8 mt + lr, k = 4 ks + lc) are loaded from shared memory once per slab
+        // instead of once per tile (those loads were 11 % of the kernel's shared wavefronts, 45 % of them bank-conflict
+        // excess: row stride P = 9)
+        constexpr bool TBW = MB & 256;
+        const int ptab = warp < 5 ? 0 : 1;
+        double afr[2][KSP];
+#pragma unroll
+        for (int mt = 0; mt < 2; ++mt)
+#pragma unroll
+          for (int ks = 0; ks < KSP; ++ks) {
+            const int kk = 4 * ks + lc;
+            afr[mt][ks] = (TBW && kk < P) ? (ptab == 0 ? sB : sG)[(8 * mt + lr) * P + kk] : 0.0;
+          }
 #pragma unroll
         for (int rr = 0; rr < (NTILE + NTH / 32 - 1) / (NTH / 32); ++rr) {
-          const int tl = warp + rr * (NTH / 32);
+          const int tl = !TBW ? warp + rr * (NTH / 32)
+                              : (warp < 5 ? (warp + 5 * rr < NB ? warp + 5 * rr : NTILE) : NB + (warp - 5) + 3 * rr);
           if (tl < NTILE) {
             const int tab = tl < NB ? 0 : tl < NB + NG ? 1 : 2;      // 0: B, 1: G, 2: Phi (warp-uniform)
             const int c0 = (tab == 0 ? tl : tab == 1 ? tl - NB : 0) * 8;
@@ -185,7 +200,7 @@ __global__ void __launch_bounds__(KB1V11Cfg<K>::NTH, MINB) kb1_v11_3d(const KB1A
                 const double b = (bok && kk < kx) ? bsrc[kk * bstride] : 0.0;
 #pragma unroll
                 for (int mt = 0; mt < 2; ++mt) {
-                  const double af = kk < kx ? X[(8 * mt + lr) * ldx + kk] : 0.0;
+                  const double af = (TBW && tab == ptab) ? afr[mt][ks] : (kk < kx ? X[(8 * mt + lr) * ldx + kk] : 0.0);
                   dmma(d[mt][0], d[mt][1], af, b);
                 }
               }

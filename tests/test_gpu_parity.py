@@ -288,7 +288,7 @@ def test_multi_material_gamma(orc):
 CANDIDATES = {1: ["v2.p1.z32", "v2.z64", "v1.z32"], 2: ["v2.z1m12e", "v2.z1m12", "v2.z2m6", "v2.p1.z2", "v1.z16"],
               3: ["v2.z2", "v2.p1.z1", "v3.z2", "v1.z8"],
               4: ["v10.wpx", "v10.w", "v10.v", "v5.r1", "v2.z1", "v1.z4"],
-              7: ["v8", "v11", "v1.z1"], 8: ["v11.mbtsie", "v11.mbtsi", "v11.mbts", "v11.mbt", "v11.mb", "v8", "v11", "v8.m1", "v1.z1m2", "v1.z1"]}
+              7: ["v8", "v11", "v1.z1"], 8: ["v11.mbtsiet", "v11.mbtsie", "v11.mbtsi", "v11.mbts", "v11.mbt", "v11.mb", "v8", "v11", "v8.m1", "v1.z1m2", "v1.z1"]}
 
 
 @pytest.mark.parametrize("k,name", [(k, n) for k, ns in CANDIDATES.items() for n in ns])

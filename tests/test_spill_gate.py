@@ -17,7 +17,7 @@ LIB = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), 
 # mangled kernel name -> (config, max STACK bytes, max registers)
 DEFAULTS = {
     "_Z10kb1_v10_3dILi4ELi0ELi0ELi33554432ELi11EEv7KB1Args": ("C4 v10.wpx", 56, 128),
-    "_Z10kb1_v11_3dILi8ELi2ELi211EEv7KB1Args": ("C5 v11.mbtsie", 0, 128),
+    "_Z10kb1_v11_3dILi8ELi2ELi467EEv7KB1Args": ("C5 v11.mbtsiet", 0, 128),
     "_Z9kb1_v2_3dILi2ELi1ELi12ELi2ELi6EEv7KB1Args": ("C3 v2.z1m12e", 40, 168),
     "_Z7kb1_p2dILi4ELi2ELi6EEv7KB1Args": ("C2 p2d.z2m6", 0, 80),
     "_Z10kb2_gatherILi3ELi8EEvPKdPKiS3_lllidPdS1_iS4_": ("KB2 3D", 0, 64),

@@ -2,7 +2,7 @@
 """One small corner-force evaluation (or integrator step) for compute-sanitizer.
 
     compute-sanitizer --tool memcheck|racecheck|synccheck python tools/sanitize.py <case>
-cases: c4 (v10.w, 3D k=4, 40 zones), c5 (v11.mbtsie, 3D k=8, 4 zones), c5v8 (v8), c3 (v2.z1m12e, 3D k=2),
+cases: c4 (v10.wpx, 3D k=4, 40 zones), c5 (v11.mbtsiet, 3D k=8, 4 zones), c5v8 (v8), c3 (v2.z1m12e, 3D k=2),
        c2 (p2d.z2m6, 2D k=4), integrator (2D k=3 RK2 step), host (pipelined host entry, 3D k=2 16^3),
        loopback (the overlap schedule of a 4-rank loopback group), p2p (2 processes, the peer-memory exchange
        over CUDA IPC, 3 evals each; compute-sanitizer follows the child processes)."""
@@ -13,7 +13,7 @@ import numpy as np
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
-CASES = {"c4": ("C4", (5, 4, 2), None, "v10.w"), "c5": ("C5", (2, 1, 2), None, "v11.mbtsie"), "c5v8": ("C5", (2, 1, 2), None, "v8"),
+CASES = {"c4": ("C4", (5, 4, 2), None, "v10.wpx"), "c5": ("C5", (2, 1, 2), None, "v11.mbtsiet"), "c5v8": ("C5", (2, 1, 2), None, "v8"),
          "c3": ("C3", (4, 4, 3), None, "v2.z1m12e"), "c2": ("C2", (9, 7), None, "p2d.z2m6")}
 
 
