@@ -158,8 +158,18 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   // stage clocks of the contraction warps (a.prof != nullptr only): sKP[s] accumulates the cycles of
   // stage s, sKP[15] holds the last stamp; written by KW thread 0 alone (PW's dt reduction uses sRed[0, 16))
   long long *sKP = reinterpret_cast<long long *>(smem + Dm::OFF_RED + 16);
+  // VMODE_ bit 5 (NOKST): the contraction warps' per-stage clock stamps compiled out (each is a runtime-checked
+  // branch at a stage barrier; the per-zone accounting of CLK stays)
+  constexpr bool KST = !(VMODE_ & 32);
+  // VMODE_ bits 6 / 7 (PFENCE, experiment): runtime-uniform, never-taken branches in the point warps' zone body
+  // (after stage C_v / before the C^T tiles) -- the contraction warps' stage stamps turned out to be scheduling
+  // fences ptxas benefits from (compiling them out: 11 % slower)
+  constexpr int PFENCE = (VMODE_ >> 6) & 3;
+  auto pfence = [&](int slot) {
+    if (a.prof != nullptr && tid == 0) sKP[12 + slot] = clock64();
+  };
   auto kstamp = [&](int slot) {
-    if (a.prof != nullptr && tid == NPW) {
+    if (KST && a.prof != nullptr && tid == NPW) {
       const long long t = clock64();
       sKP[slot] += t - sKP[15];
       sKP[15] = t;
@@ -647,6 +657,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       ea = fma(tPhi[q0a * T + j0], ue, ea);
       eb = fma(tPhi[(q0a + NH) * T + j0], ue, eb);
     }
+    if (PFENCE & 1) pfence(0);
     double Ja[3][3], Gva[3][3], Jb[3][3], Gvb[3][3];
 #pragma unroll
     for (int c = 0; c < 3; ++c)
@@ -706,6 +717,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
       for (int cd = 0; cd < 9; ++cd) acc += oa.S[cd / 3][cd % 3] + ob.S[cd / 3][cd % 3];
       if (acc == 1.2345e300) jb[Dm::O_PQ + sa] = acc;
     } else if (PCT) {
+      if (PFENCE & 2) pfence(1);
       static_assert(N == 8 && P <= 8 && T <= 8 && NPW == 256, "PCT: one m8n8k4 tile per (warp, field), k-steps = q0 halves");
       const int ln = tid & 31, lr = ln >> 2, lc = ln & 3;   // lr = q1, lc = q0a (pr = tid)
       // A fragments: table^T[a = lr][q0 = 4 s + lc] (rows a >= P / T are zero)
