@@ -165,6 +165,9 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   // (after stage C_v / before the C^T tiles) -- the contraction warps' stage stamps turned out to be scheduling
   // fences ptxas benefits from (compiling them out: 11 % slower)
   constexpr int PFENCE = (VMODE_ >> 6) & 3;
+  // VMODE_ bits 8 / 9 (KFENCE, experiment): a never-taken stamp branch between the work blocks of the forward
+  // stages A, B (bit 8) and C_x (bit 9), so ptxas does not interleave the blocks' loads
+  constexpr int KFENCE = (VMODE_ >> 8) & 3;
   auto pfence = [&](int slot) {
     if (a.prof != nullptr && tid == 0) sKP[12 + slot] = clock64();
   };
@@ -256,6 +259,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
 #pragma unroll
     for (int blk = 0; blk < (SKAB ? 0 : (6 * P2 + T2 + NKW - 1) / NKW); ++blk) {
       const int r = r0_ + blk * NKW;
+      if ((KFENCE & 1) && blk > 0) kstamp(14);
       const CTZ<K> C{zc * (blk + 1)};
       if (r < 6 * P2 + T2) {
       if (r < 6 * P2) {
@@ -300,6 +304,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
 #pragma unroll
     for (int blk = 0; blk < (SKAB ? 0 : (6 * N * P + N * T + NKW - 1) / NKW); ++blk) {
       const int r = (bal && blk == 1) ? (r0_ >= NB ? NKW + r0_ - NB : NB + NU) : r0_ + blk * NKW;
+      if ((KFENCE & 1) && blk > 0) kstamp(14);
       const CTZ<K> C{zc * (blk + 1)};
       if (r < 6 * N * P + N * T) {
       if (r < 6 * N * P) {
@@ -348,6 +353,7 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
 #pragma unroll
     for (int blk = 0; blk < (SKCX ? 0 : (9 * N2 + NKW - 1) / NKW); ++blk) {
       const int r = r0_ + blk * NKW;
+      if ((KFENCE & 2) && blk > 0) kstamp(14);
       const CTZ<K> C{zc * (blk + 1)};
       if (r < 9 * N2) {
       const int cm = r / N2, col = r - cm * N2;   // cm is warp-uniform (N2 = 64)
