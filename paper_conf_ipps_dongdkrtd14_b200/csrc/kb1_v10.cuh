@@ -168,6 +168,9 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
   // VMODE_ bits 8 / 9 (KFENCE, experiment): a never-taken stamp branch between the work blocks of the forward
   // stages A, B (bit 8) and C_x (bit 9), so ptxas does not interleave the blocks' loads
   constexpr int KFENCE = (VMODE_ >> 8) & 3;
+  // VMODE_ bit 10 (FBM): forward stage B on DMMA instead of DFMA + LDCU (the C5 lesson)
+  constexpr bool FBM = VMODE_ & 1024;
+  constexpr bool PADU_ = (OPT & 128) != 0;
   auto pfence = [&](int slot) {
     if (a.prof != nullptr && tid == 0) sKP[12 + slot] = clock64();
   };
@@ -297,6 +300,63 @@ __global__ void __launch_bounds__(KB1V5Cfg<K, MODE>::NTH, 1) kb1_v10_3d(const KB
     kstamp(8);
     // stage B: a1 -> q1; position fields -> UX (scratch), velocity fields + e -> ub
     // (BAL: the second block's e items go to the threads without a field item, not to threads 0-15 again)
+    if (FBM) {   // VMODE_ bit 10: stage B on DMMA (kb1_v5.cuh's form): M = q1, K = a1 (P padded to 8), N = (f, q2, a0)
+      static_assert(!FBM || (!PADU_ && N == 8), "FBM: the natural U layout, one m-tile of q1");
+      const int kt = opaque_tid() - NPW, kwarp = kt >> 5, lr = (kt & 31) >> 2, lc = kt & 3;
+      constexpr int KS_P = (P + 3) / 4, KS_T = (T + 3) / 4;
+      double fB[KS_P], fG[KS_P], fP[KS_T];
+#pragma unroll
+      for (int s2 = 0; s2 < KS_P; ++s2) {
+        fB[s2] = tfrag<false>(tB, P, N, P, lr, 4 * s2 + lc);
+        fG[s2] = tfrag<false>(tG, P, N, P, lr, 4 * s2 + lc);
+      }
+#pragma unroll
+      for (int s2 = 0; s2 < KS_T; ++s2) fP[s2] = tfrag<false>(tPhi, T, N, T, lr, 4 * s2 + lc);
+      constexpr int NC = 6 * N * P, NTL = (NC + 7) / 8, JPWT = (NTL + NKWW - 1) / NKWW;
+#pragma unroll
+      for (int t = 0; t < JPWT; ++t) {
+        const int j = kwarp + t * NKWW;
+        const int nb = min(j * 8 + lr, NC - 1);
+        const int fb = nb / (N * P), rb = nb - fb * (N * P), q2b = rb / P, a0b = rb - q2b * P;
+        const double *TBb = Tr + Dm::O_T + ((fb * 2 + 0) * N + q2b) * P2 + a0b;
+        double u[3][2] = {{0.0, 0.0}, {0.0, 0.0}, {0.0, 0.0}};
+#pragma unroll
+        for (int s2 = 0; s2 < KS_P; ++s2) {
+          const int a1 = min(4 * s2 + lc, P - 1);
+          const double tb = TBb[a1 * P], tg = TBb[N * P2 + a1 * P];
+          dmma(u[0][0], u[0][1], fB[s2], tb);
+          dmma(u[1][0], u[1][1], fG[s2], tb);
+          dmma(u[2][0], u[2][1], fB[s2], tg);
+        }
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+          const int n = j * 8 + 2 * lc + i;
+          if (j < NTL && n < NC) {
+            const int f = n / (N * P), rr = n - f * (N * P), q2 = rr / P, a0 = rr - q2 * P;
+            double *U = (f < 3 ? UX + f * 3 * UM : ub + (f - 3) * 3 * UM) + q2 * UQ + lr * UQ1 + a0;
+            U[0] = u[0][i];
+            U[UM] = u[1][i];
+            U[2 * UM] = u[2][i];
+          }
+        }
+      }
+      constexpr int NCE = N * T, NTE = (NCE + 7) / 8;   // UE = Phi . TE
+      for (int te = kwarp; te < NTE; te += NKWW) {
+        const int nb = min(te * 8 + lr, NCE - 1);
+        const int q2b = nb / T, j0b = nb - q2b * T;
+        double d0 = 0.0, d1 = 0.0;
+#pragma unroll
+        for (int s2 = 0; s2 < KS_T; ++s2) dmma(d0, d1, fP[s2], Tr[Dm::O_TE + q2b * T2 + min(4 * s2 + lc, T - 1) * T + j0b]);
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+          const int n = te * 8 + 2 * lc + i;
+          if (n < NCE) {
+            const int q2 = n / T, j0 = n - q2 * T;
+            ub[Dm::O_UE + q2 * UQE + lr * T + j0] = i ? d1 : d0;
+          }
+        }
+      }
+    } else
     {
     const int r0_ = opaque_tid() - NPW;
     constexpr int NB = 6 * N * P, NU = N * T;
