@@ -323,6 +323,11 @@ KB1Variant select_variant(int dim, int k, bool need_point_j0) {
       if (strcmp(force, "v10.wpxu") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | 128, 3 | 8>(); d.name = "v10.wpxu"; return d; }
       if (strcmp(force, "v10.wpxn") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | 2048, 3 | 8>(); d.name = "v10.wpxn"; return d; }
       if (strcmp(force, "v10.wpxb2") == 0) { d = variant3v10<4, 0, 0, (1 << 25), 3 | 8 | 1024>(); d.name = "v10.wpxb2"; return d; }
+      if (strcmp(force, "v10.wpxbulk") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | 1, 3 | 8>(); d.name = "v10.wpxbulk"; return d; }
+      if (strcmp(force, "v10.wpxlate") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | 2, 3 | 8>(); d.name = "v10.wpxlate"; return d; }
+      if (strcmp(force, "v10.wpxv16") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | 16, 3 | 8>(); d.name = "v10.wpxv16"; return d; }
+      if (strcmp(force, "v10.wpxspread") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | 64, 3 | 8>(); d.name = "v10.wpxspread"; return d; }
+      if (strcmp(force, "v10.wpxbal") == 0) { d = variant3v10<4, 0, 0, (1 << 25) | 4, 3 | 8>(); d.name = "v10.wpxbal"; return d; }
       if (strcmp(force, "v10.d2") == 0) { d = variant3v10<4, 2>(); d.name = "v10.d2"; return d; }
       if (strcmp(force, "v5.r2") == 0) { d = variant3v5<4, 0, 2>(); d.name = "v5.r2"; return d; }
       if (strcmp(force, "v5.r1d1") == 0) { d = variant3v5<4, 1, 1>(); d.name = "v5.r1d1"; return d; }
