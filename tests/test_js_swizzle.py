@@ -42,3 +42,18 @@ def test_row_pair_accesses():
         for pair in range(4):
             slots = [(js_idx(c, 2 * pair) % 16) // 2 for c in range(c0, c0 + 8)]
             assert len(set(slots)) == 8
+
+
+def test_pct_y_slots_stay_in_the_warps_own_rows():
+    """v10.wpx (PCT): point warp q2 stores Y[cd][a0][q1] at plane cd, slot q2*N^2 + a0*N + q1 (YE: j0 < 4) over J, and
+    relies on every J slot of those rows belonging to its own points (lane l: q1 = l >> 2, q0 = l & 3 and l & 3 + 4),
+    so no other warp's J is overwritten; the contraction warps' B^T reads the same slots."""
+    for q2 in range(N):
+        own = {js_idx(q2 * N + (l >> 2), (l & 3) + s) for l in range(32) for s in (0, 4)}
+        assert own == set(range(q2 * N * N, (q2 + 1) * N * N))          # the warp's points fill its 64 slots
+        ys = {q2 * N * N + a0 * N + q1 for a0 in range(5) for q1 in range(N)}
+        assert ys <= own                                                   # Y (a0 < 5) only over its own J
+        # the m8n8k4 store pattern: lane (lr = a0, lc) writes q1 = 2 lc, 2 lc + 1 -> 16-byte aligned pairs
+        for lr in range(5):
+            for lc in range(4):
+                assert (q2 * N * N + lr * N + 2 * lc) % 2 == 0
